@@ -1,0 +1,184 @@
+/*
+ * madpipe.h -- C ABI of the B200-native MadPipe-DP hot path (libmadpipe.so).
+ *
+ * The library decides, for a chain of L DNN layers, P GPUs of memory M and
+ * links of bandwidth beta, the smallest candidate period tau for which the
+ * memory-aware dynamic program of MadPipe (Beaumont, Eyraud-Dubois, Shilova,
+ * hal-03025305, section 4.2) finds an allocation, and returns that allocation.
+ * It is the "first phase" of MadPipe (Algorithm 1) with the serial
+ * binary search replaced by a batched sweep over candidate periods (DESIGN.md
+ * reading Q1/Q14).  "P:n" = line n of the paper text; "Qn" = DESIGN.md readings.
+ *
+ * Problem statement mirrored by the ABI: "finding a good load
+ * balancing ... on P given processors with memory capacity M and connected via
+ * the network with bandwidth beta".
+ *
+ * Conventions for every entry point
+ *   - Return 0 (MADPIPE_OK) on success, 1 (MADPIPE_INFEASIBLE) when no candidate
+ *     period admits an allocation (a valid outcome, not an error), negative on
+ *     error; madpipe_last_error() then describes it.
+ *   - Pointers marked [host] are host memory, [dev] are device memory on the
+ *     ctx's device.  Input arrays are read-only and owned by the caller; the
+ *     library keeps no pointer after return.  Output arrays are caller-allocated.
+ *   - All entry points are synchronous with respect to the host (they return
+ *     after their GPU work is complete) unless stated otherwise.
+ *   - One ctx per host thread; a ctx is bound to one CUDA device.
+ *   - Arithmetic is IEEE binary64 without FMA contraction; memory is int64
+ *     bytes.  Results are bit-identical to the plain CPU oracle (oracle/).
+ */
+#ifndef MADPIPE_H
+#define MADPIPE_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MADPIPE_OK          0
+#define MADPIPE_INFEASIBLE  1
+#define MADPIPE_EINVAL    (-1)   /* invalid argument (see madpipe_validate)            */
+#define MADPIPE_ENOMEM    (-2)   /* device or host allocation failed                    */
+#define MADPIPE_ECUDA     (-3)   /* CUDA runtime error (no device, launch failure, ...) */
+#define MADPIPE_ESTATE    (-5)   /* call out of order (e.g. resolve of an infeasible j) */
+
+/* A linear (or linearised) chain of L layers (section 3).
+ *   uF[L], uB[L] : forward / backward duration of layer i+1 on one mini-batch,
+ *                  seconds; finite, >= 0, uF+uB > 0 (reading Q9).
+ *   W[L]         : weight bytes of layer i+1 (>= 0); a GPU holding it stores 3 W.
+ *   a[L+1]       : activation bytes; a[0] = network input a^(0), a[l] = output of F_l
+ *                  (reading Q5).  a_l is also the size of b^(l).
+ * Pointers are [host] for madpipe_solve / _candidates / _dp_table / _solve_batch,
+ * [dev] for madpipe_solve_dev, and either for madpipe_sweep / _resolve (the
+ * library asks the CUDA runtime which; device arrays are not value-checked). */
+typedef struct {
+    int32_t L;
+    const double  *uF;
+    const double  *uB;
+    const int64_t *W;
+    const int64_t *a;
+} madpipe_chain;
+
+/* Range of the delay grid V (reading Q8). PAPER: 0..U(1,L)+sum C,
+ * a delay beyond the range makes the transition infeasible.  SAFE:
+ * 0..2(U(1,L)+sum C)+tau, saturating at the top level. */
+typedef enum { MADPIPE_VRANGE_PAPER = 0, MADPIPE_VRANGE_SAFE = 1 } madpipe_vrange;
+
+/* Discretisation (the paper uses 11 memory levels and 51 delay levels). */
+typedef struct {
+    int32_t n_mem;      /* levels of the special GPU's memory m_P in [0,M], 2..64       */
+    int32_t n_delay;    /* levels of the delay V, 2..65535                               */
+    int32_t n_periods;  /* candidate periods, uniform on [lb, ub] (P:205 l.1-2, Q14), >= 1 */
+    int32_t v_range;    /* madpipe_vrange                                                 */
+    int32_t early_exit; /* 0: evaluate every candidate; 1: stop at the first feasible one  */
+} madpipe_disc;
+
+/* Result of a solve (the decisions along the optimal path give the
+ * partitioning and the assignment).  Stages are in chain order; stage_proc is
+ * in [0, P-2] for the normal GPUs (numbered in chain order) and P-1 for the
+ * special GPU.  The three stage arrays are caller-allocated with
+ * capacity L; the library writes n_stages entries. */
+typedef struct {
+    double   period;        /* tau_{j*}: the candidate period found (Alg. 1 step 5, Q16)   */
+    double   load_period;   /* load of the most loaded GPU or link, <= period       */
+    double   special_load;  /* DP root value A[L][P-1][0][0]: the special GPU's load         */
+    int32_t  cand_index;    /* j* (or -1 if infeasible)                                      */
+    int32_t  n_stages;
+    int32_t *stage_first;   /* [host] capacity L, 1-based first layer                        */
+    int32_t *stage_last;    /* [host] capacity L, 1-based last layer                         */
+    int32_t *stage_proc;    /* [host] capacity L                                              */
+    int64_t  cell_updates;  /* relaxations evaluated by the sweep             */
+} madpipe_alloc;
+
+typedef struct madpipe_ctx madpipe_ctx;
+
+/* ---- context --------------------------------------------------------------
+ * Create a ctx on CUDA device `device`.  `cuda_stream` is a cudaStream_t to
+ * issue work on (e.g. torch.cuda.current_stream().cuda_stream), or NULL for a
+ * stream owned by the ctx.  `mem_budget` bounds the device bytes used for DP
+ * tables (0 = 60% of the free memory at creation).  Returns MADPIPE_ECUDA if
+ * no device is usable. */
+int  madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stream, int64_t mem_budget);
+void madpipe_ctx_destroy(madpipe_ctx *ctx);
+const char *madpipe_last_error(const madpipe_ctx *ctx);   /* ctx may be NULL */
+
+/* ---- host-only helpers (no GPU needed) ------------------------------------ */
+/* Check every argument rule of this header; MADPIPE_OK or MADPIPE_EINVAL.
+ * Rules: L >= 1; P >= 1; M > 0; beta > 0 and not NaN (beta = +inf allowed:
+ * C = 0); uF, uB finite, >= 0, uF+uB > 0; W >= 0; a >= 0; 2 <= n_mem <= 64;
+ * 2 <= n_delay <= 65535; n_periods >= 1; v_range in {0,1}; int64 overflow
+ * guards 3*sum W + (g_max)*sum a and (M-1) + (n_mem-1)*(3 sum W + g_max sum a). */
+int madpipe_validate(const madpipe_chain *chain, int32_t P, int64_t M, double beta,
+                     const madpipe_disc *disc);
+/* Candidates owned by `rank` of `world` (interleaved: j = rank, rank+world, ...;
+ * DESIGN.md 7).  Writes up to n_periods indices into out[] and their count. */
+int madpipe_shard(int32_t n_periods, int32_t rank, int32_t world, int32_t *out, int32_t *count);
+/* Exact number of cell-updates of candidate period tau:
+ * sum_l (l - kmin(l) + 1) (P-1) n_delay n_mem, where kmin(l) is the smallest k
+ * with U(k,l) <= tau.  [host] chain. */
+int64_t madpipe_cell_updates(const madpipe_chain *chain, int32_t P, const madpipe_disc *disc,
+                             double tau);
+
+/* ---- the hot path -----------------------------------------------------------
+ * Full solve on one GPU (world = 1): profile prep (a1), candidate grid (a2),
+ * the batched wavefront DP over every candidate (a3-a5), root test and
+ * minimum (a6), winner re-solve and device traceback (a8), result (a9).
+ * [host] chain and output. */
+int madpipe_solve(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                  double beta, const madpipe_disc *disc, madpipe_alloc *out);
+/* Same, with the chain arrays already resident in device memory ([dev]). */
+int madpipe_solve_dev(madpipe_ctx *ctx, const madpipe_chain *chain_dev, int32_t P, int64_t M,
+                      double beta, const madpipe_disc *disc, madpipe_alloc *out);
+
+/* Multi-GPU building blocks (one process per GPU).
+ * madpipe_sweep evaluates this rank's shard of candidates and writes the
+ * smallest feasible candidate index it owns (INT32_MAX if none) to *j_local
+ * [dev, int32]; the caller min-reduces it across ranks (one NCCL all-reduce,
+ * a7) and passes the global minimum to madpipe_resolve [dev, int32], which
+ * re-solves that candidate and traces it back; every rank gets the same result.
+ * cell_updates_out [host] receives this rank's relaxation count. With
+ * disc->early_exit the rank stops at its first feasible candidate. */
+int madpipe_sweep(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                  double beta, const madpipe_disc *disc, int32_t rank, int32_t world,
+                  int32_t *j_local, int64_t *cell_updates_out);
+int madpipe_resolve(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                    double beta, const madpipe_disc *disc, const int32_t *j_star,
+                    madpipe_alloc *out);
+
+/* Batch of n independent chains (BASELINE config 5) with per-chain P[i],
+ * M[i], beta[i] and a shared discretisation; out[i] as for madpipe_solve.
+ * All (chain, candidate) pairs run as one sweep. Returns MADPIPE_OK if the call
+ * succeeded (each out[i].cand_index is -1 for an infeasible chain). [host]. */
+int madpipe_solve_batch(madpipe_ctx *ctx, int32_t n, const madpipe_chain *chains,
+                        const int32_t *P, const int64_t *M, const double *beta,
+                        const madpipe_disc *disc, madpipe_alloc *out);
+
+/* ---- parity / debug exports (small configs) ------------------------------- */
+/* Every candidate's period tau_out[n_periods] and root value root_out[n_periods]
+ * (A_j[L][P-1][0][0]; +inf if infeasible). [host]. */
+int madpipe_candidates(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                       double beta, const madpipe_disc *disc, double *tau_out, double *root_out);
+/* Full DP table of candidate j, A_out[(L+1)*P*n_delay*n_mem] in [l][p][v][m]
+ * order, and the decision arg_out (same shape, may be NULL): 2k+o with o = 1
+ * for the special GPU, -1 where the cell is infeasible (tie-break Q11). [host]. */
+int madpipe_dp_table(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                     double beta, const madpipe_disc *disc, int32_t j, double *A_out,
+                     int32_t *arg_out);
+
+/* Timing of the last solve/sweep on the ctx's stream (CUDA events): total
+ * milliseconds of the sweep kernels, of the dominant step kernel alone, and
+ * the number of kernel launches issued. */
+int madpipe_last_timing(const madpipe_ctx *ctx, double *sweep_ms, double *step_kernel_ms,
+                        int64_t *launches);
+/* per_launch = 1: bracket every step-kernel launch with CUDA events so that
+ * madpipe_last_timing reports the step kernel's own time (bench roofline);
+ * 0 (default): only the sweep is timed. */
+int madpipe_set_timing(madpipe_ctx *ctx, int per_launch);
+/* Bytes the last call copied host->device and device->host (inputs, job
+ * descriptors, results); for the bench's end-to-end record. */
+int madpipe_last_io(const madpipe_ctx *ctx, int64_t *h2d_bytes, int64_t *d2h_bytes);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MADPIPE_H */

@@ -210,27 +210,34 @@ static int64_t fill_table(const chain_t *c, double tau, double *A, int32_t *ARG)
         int kmin = kmin_of(c, tau, l);
         if (P > 1 && kmin <= l)
             updates += (int64_t)(l - kmin + 1) * (P - 1) * n_v * n_m;
-        for (int p = 1; p < P; p++) {
-            for (int v = 0; v < n_v; v++) {
+        /* For each delay level v, the options k = kmin..l are scanned in
+         * ascending order (N before S) for every cell (p, m) of the row; the
+         * transition of (k, l, v) does not depend on (p, m), so it is computed
+         * once per k.  Each cell still sees its options in the order of O6. */
+        for (int v = 0; v < n_v; v++) {
+            for (int p = 1; p < P; p++)
                 for (int m = 0; m < n_m; m++) {
-                    double best = INFINITY;
-                    int32_t arg = -1;
-                    for (int k = kmin; k <= l; k++) {
-                        trans_t t = transition(c, tau, dV, k, l, v);
-                        if (k > 1 && (t.vn == VN_OVERFLOW || c->C[k - 1] > tau)) continue;
+                    A[IDX(c, l, p, v, m)] = INFINITY;
+                    if (ARG) ARG[IDX(c, l, p, v, m)] = -1;
+                }
+            for (int k = kmin; k <= l; k++) {
+                trans_t t = transition(c, tau, dV, k, l, v);
+                if (k > 1 && (t.vn == VN_OVERFLOW || c->C[k - 1] > tau)) continue;
+                double Ukl = U(c, k, l);
+                for (int p = 1; p < P; p++) {
+                    for (int m = 0; m < n_m; m++) {
+                        double *best = &A[IDX(c, l, p, v, m)];
                         /* T_N: stage k..l on a normal processor */
                         if (t.nf) {
                             double cand = A[IDX(c, k - 1, p - 1, t.vn, m)];
-                            if (cand < best) { best = cand; arg = 2 * k; }
+                            if (cand < *best) { *best = cand; if (ARG) ARG[IDX(c, l, p, v, m)] = 2 * k; }
                         }
                         /* T_S: stage k..l on the special processor */
                         if ((int64_t)m + t.d <= (int64_t)(n_m - 1)) {
-                            double cand = U(c, k, l) + A[IDX(c, k - 1, p, t.vn, m + (int)t.d)];
-                            if (cand <= tau && cand < best) { best = cand; arg = 2 * k + 1; }
+                            double cand = Ukl + A[IDX(c, k - 1, p, t.vn, m + (int)t.d)];
+                            if (cand <= tau && cand < *best) { *best = cand; if (ARG) ARG[IDX(c, l, p, v, m)] = 2 * k + 1; }
                         }
                     }
-                    A[IDX(c, l, p, v, m)] = best;
-                    if (ARG) ARG[IDX(c, l, p, v, m)] = arg;
                 }
             }
         }

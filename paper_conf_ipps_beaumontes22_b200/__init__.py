@@ -1,0 +1,188 @@
+"""B200-native MadPipe-DP hot path (Beaumont, Eyraud-Dubois, Shilova, hal-03025305).
+
+Thin Python layer over the C ABI of ``libmadpipe.so`` (include/madpipe.h): the
+memory-aware dynamic program of MadPipe section 4.2 evaluated over a batched
+sweep of candidate periods (replacing Algorithm 1's serial search),
+with a device-side traceback.  PyTorch is used only for device memory, streams
+and process groups (see ``distributed.py``).  There is no CPU fallback.
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+
+from . import _native as N
+from ._native import VRANGE_PAPER, VRANGE_SAFE, MadpipeError  # noqa: F401
+
+__all__ = ["Context", "validate", "shard", "cell_updates", "VRANGE_PAPER", "VRANGE_SAFE",
+           "MadpipeError"]
+
+
+def validate(chain, P, M, beta, n_mem, n_delay, n_periods, v_range=VRANGE_PAPER) -> int:
+    """madpipe_validate (host only): 0 or -1 (EINVAL)."""
+    hc = N.HostChain(chain)
+    d = N.make_disc(n_mem, n_delay, n_periods, v_range)
+    return N.lib().madpipe_validate(ctypes.byref(hc.c), int(P), int(M), float(beta), ctypes.byref(d))
+
+
+def shard(n_periods, rank, world):
+    """madpipe_shard (host only): the candidate indices owned by a rank."""
+    out = np.zeros(max(1, n_periods), np.int32)
+    cnt = ctypes.c_int32()
+    N.check(N.lib().madpipe_shard(n_periods, rank, world, out.ctypes.data_as(N._i32p), ctypes.byref(cnt)))
+    return [int(x) for x in out[:cnt.value]]
+
+
+def cell_updates(chain, P, n_mem, n_delay, tau) -> int:
+    hc = N.HostChain(chain)
+    d = N.make_disc(n_mem, n_delay, 1)
+    return int(N.lib().madpipe_cell_updates(ctypes.byref(hc.c), int(P), ctypes.byref(d), float(tau)))
+
+
+class _DevChain:
+    def __init__(self, d):
+        self.L = int(d["uF"].numel())
+        self.keep = d
+        self.c = N.Chain(self.L, d["uF"].data_ptr(), d["uB"].data_ptr(), d["W"].data_ptr(),
+                         d["a"].data_ptr())
+
+
+def _any_chain(chain):
+    if hasattr(chain["uF"], "is_cuda") and chain["uF"].is_cuda:
+        return _DevChain(chain)
+    return N.HostChain(chain)
+
+
+class Context:
+    """A libmadpipe context bound to one CUDA device (madpipe_ctx_create)."""
+
+    def __init__(self, device: int = 0, stream=None, mem_budget: int = 0):
+        self._lib = N.lib()
+        h = ctypes.c_void_p()
+        rc = self._lib.madpipe_ctx_create(ctypes.byref(h), int(device),
+                                          ctypes.c_void_p(stream) if stream else None, int(mem_budget))
+        if rc != N.OK:
+            raise MadpipeError(rc, N.last_error(None))
+        self.h = h
+        self.device = device
+
+    def close(self):
+        if getattr(self, "h", None):
+            self._lib.madpipe_ctx_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    # ------------------------------------------------------------------ hot path
+    def solve(self, chain, P, M, beta, n_mem, n_delay, n_periods, v_range=VRANGE_PAPER,
+              early_exit=False):
+        hc = N.HostChain(chain)
+        d = N.make_disc(n_mem, n_delay, n_periods, v_range, early_exit)
+        buf = N.AllocBuf(hc.L)
+        rc = self._lib.madpipe_solve(self.h, ctypes.byref(hc.c), int(P), int(M), float(beta),
+                                     ctypes.byref(d), ctypes.byref(buf.s))
+        N.check(rc, self.h)
+        return buf.result(rc)
+
+    def solve_dev(self, dchain, P, M, beta, n_mem, n_delay, n_periods, v_range=VRANGE_PAPER,
+                  early_exit=False):
+        """``dchain``: dict of CUDA tensors uF, uB (float64), W, a (int64) on this device."""
+        L = int(dchain["uF"].numel())
+        c = N.Chain(L, dchain["uF"].data_ptr(), dchain["uB"].data_ptr(), dchain["W"].data_ptr(),
+                    dchain["a"].data_ptr())
+        d = N.make_disc(n_mem, n_delay, n_periods, v_range, early_exit)
+        buf = N.AllocBuf(L)
+        rc = self._lib.madpipe_solve_dev(self.h, ctypes.byref(c), int(P), int(M), float(beta),
+                                         ctypes.byref(d), ctypes.byref(buf.s))
+        N.check(rc, self.h)
+        return buf.result(rc)
+
+    def sweep(self, chain, P, M, beta, n_mem, n_delay, n_periods, rank, world, j_local_ptr,
+              v_range=VRANGE_PAPER, early_exit=False) -> int:
+        """Evaluate this rank's candidates; writes the local minimum feasible index
+        (INT32_MAX if none) to the int32 device buffer at ``j_local_ptr``.  ``chain``
+        is a host dict of arrays or a dict of CUDA tensors."""
+        hc = _any_chain(chain)
+        d = N.make_disc(n_mem, n_delay, n_periods, v_range, early_exit)
+        cu = ctypes.c_int64()
+        N.check(self._lib.madpipe_sweep(self.h, ctypes.byref(hc.c), int(P), int(M), float(beta),
+                                        ctypes.byref(d), int(rank), int(world),
+                                        ctypes.c_void_p(j_local_ptr), ctypes.byref(cu)), self.h)
+        return cu.value
+
+    def resolve(self, chain, P, M, beta, n_mem, n_delay, n_periods, j_star_ptr,
+                v_range=VRANGE_PAPER):
+        hc = _any_chain(chain)
+        d = N.make_disc(n_mem, n_delay, n_periods, v_range)
+        buf = N.AllocBuf(hc.L)
+        rc = self._lib.madpipe_resolve(self.h, ctypes.byref(hc.c), int(P), int(M), float(beta),
+                                       ctypes.byref(d), ctypes.c_void_p(j_star_ptr), ctypes.byref(buf.s))
+        N.check(rc, self.h)
+        return buf.result(rc)
+
+    def solve_batch(self, chains, Ps, Ms, betas, n_mem, n_delay, n_periods, v_range=VRANGE_PAPER,
+                    early_exit=False):
+        hcs = [N.HostChain(c) for c in chains]
+        n = len(hcs)
+        arr = (N.Chain * n)(*[h.c for h in hcs])
+        P = np.ascontiguousarray(Ps, np.int32)
+        M = np.ascontiguousarray(Ms, np.int64)
+        B = np.ascontiguousarray(betas, np.float64)
+        bufs = [N.AllocBuf(h.L) for h in hcs]
+        outs = (N.Alloc * n)(*[b.s for b in bufs])
+        d = N.make_disc(n_mem, n_delay, n_periods, v_range, early_exit)
+        N.check(self._lib.madpipe_solve_batch(self.h, n, arr, P.ctypes.data_as(N._i32p),
+                                              M.ctypes.data_as(N._i64p), B.ctypes.data_as(N._dp),
+                                              ctypes.byref(d), outs), self.h)
+        res = []
+        for b, o in zip(bufs, outs):
+            b.s = o
+            res.append(b.result(N.OK if o.cand_index >= 0 else N.INFEASIBLE))
+        return res
+
+    # ------------------------------------------------------------------ parity exports
+    def candidates(self, chain, P, M, beta, n_mem, n_delay, n_periods, v_range=VRANGE_PAPER):
+        hc = N.HostChain(chain)
+        d = N.make_disc(n_mem, n_delay, n_periods, v_range)
+        tau = np.empty(n_periods)
+        root = np.empty(n_periods)
+        N.check(self._lib.madpipe_candidates(self.h, ctypes.byref(hc.c), int(P), int(M), float(beta),
+                                             ctypes.byref(d), tau.ctypes.data_as(N._dp),
+                                             root.ctypes.data_as(N._dp)), self.h)
+        return tau, root
+
+    def dp_table(self, chain, P, M, beta, n_mem, n_delay, n_periods, j, v_range=VRANGE_PAPER,
+                 with_arg=True):
+        hc = N.HostChain(chain)
+        d = N.make_disc(n_mem, n_delay, n_periods, v_range)
+        A = np.empty((hc.L + 1, P, n_delay, n_mem), np.float64)
+        ARG = np.empty((hc.L + 1, P, n_delay, n_mem), np.int32) if with_arg else None
+        N.check(self._lib.madpipe_dp_table(self.h, ctypes.byref(hc.c), int(P), int(M), float(beta),
+                                           ctypes.byref(d), int(j), A.ctypes.data_as(N._dp),
+                                           ARG.ctypes.data_as(N._i32p) if with_arg else None),
+                self.h)
+        return A, ARG
+
+    def set_timing(self, per_launch: bool):
+        N.check(self._lib.madpipe_set_timing(self.h, 1 if per_launch else 0), self.h)
+
+    def last_io(self):
+        a = ctypes.c_int64(); b = ctypes.c_int64()
+        N.check(self._lib.madpipe_last_io(self.h, ctypes.byref(a), ctypes.byref(b)))
+        return dict(h2d_bytes=a.value, d2h_bytes=b.value)
+
+    def last_timing(self):
+        s = ctypes.c_double(); k = ctypes.c_double(); n = ctypes.c_int64()
+        N.check(self._lib.madpipe_last_timing(self.h, ctypes.byref(s), ctypes.byref(k), ctypes.byref(n)))
+        return dict(sweep_ms=s.value, step_ms=k.value, launches=n.value)

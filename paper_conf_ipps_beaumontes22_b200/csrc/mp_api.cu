@@ -1,0 +1,792 @@
+// mp_api.cu -- C ABI of libmadpipe (include/madpipe.h): validation, device
+// memory, the batched candidate sweep engine, winner re-solve and traceback.
+//
+// Every step of the DP path runs in the kernels of mp_kernels.cu; this file
+// only validates arguments, moves the O(L) profile to the device, lays out the
+// DP tables in HBM and issues the launches (DESIGN.md sections 6-7).
+#include <algorithm>
+#include <chrono>
+#include <climits>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "../../include/madpipe.h"
+#include "mp_internal.cuh"
+
+using namespace mp;
+
+struct DevBuf {
+    void *p = nullptr;
+    size_t n = 0;
+    cudaError_t ensure(size_t bytes) {
+        if (bytes <= n) return cudaSuccess;
+        if (p) cudaFree(p);
+        p = nullptr; n = 0;
+        size_t want = std::max(bytes, (size_t)256);
+        cudaError_t e = cudaMalloc(&p, want);
+        if (e == cudaSuccess) n = want;
+        return e;
+    }
+    void release() { if (p) cudaFree(p); p = nullptr; n = 0; }
+};
+
+struct madpipe_ctx {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    int64_t mem_budget = 0;
+    std::string err;
+    DevBuf tables, jobs, tiles, chains, chain_data, jl, counts, roots, trace, stages, scratch;
+    cudaEvent_t ev_a = nullptr, ev_b = nullptr;
+    double sweep_ms = 0.0, step_ms = 0.0;
+    int64_t launches = 0;
+    int64_t h2d_bytes = 0, d2h_bytes = 0;
+    int per_launch_timing = 0;
+    std::vector<cudaEvent_t> ev_pool;
+};
+
+static thread_local std::string g_err;
+
+static int fail(madpipe_ctx *ctx, int code, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (ctx) ctx->err = buf;
+    g_err = buf;
+    return code;
+}
+
+#define CUDA_TRY(ctx, expr)                                                                   \
+    do {                                                                                      \
+        cudaError_t _e = (expr);                                                              \
+        if (_e != cudaSuccess)                                                                \
+            return fail(ctx, _e == cudaErrorMemoryAllocation ? MADPIPE_ENOMEM : MADPIPE_ECUDA, \
+                        "%s: %s (%s:%d)", #expr, cudaGetErrorString(_e), __FILE__, __LINE__); \
+    } while (0)
+
+// All host<->device traffic of the library goes through these two counters
+// (reported by madpipe_last_io for the bench's e2e record).
+static cudaError_t h2d(madpipe_ctx *ctx, void *dst, const void *src, size_t bytes) {
+    ctx->h2d_bytes += (int64_t)bytes;
+    return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, ctx->stream);
+}
+static cudaError_t d2h(madpipe_ctx *ctx, void *dst, const void *src, size_t bytes) {
+    ctx->d2h_bytes += (int64_t)bytes;
+    return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToHost, ctx->stream);
+}
+
+static int fill_int_max(madpipe_ctx *ctx, int32_t *dev, size_t n) {
+    std::vector<int32_t> h(n, INT32_MAX);
+    CUDA_TRY(ctx, h2d(ctx, dev, h.data(), sizeof(int32_t) * n));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    return MADPIPE_OK;
+}
+
+static int nmp_of(int n_m) {
+    int n = 2;
+    while (n < n_m) n <<= 1;
+    return n;
+}
+
+// ---------------------------------------------------------------------------
+// host-only helpers
+// ---------------------------------------------------------------------------
+static int validate_impl(const madpipe_chain *ch, int32_t P, int64_t M, double beta,
+                         const madpipe_disc *disc, bool host_arrays, std::string *why) {
+    auto bad = [&](const char *msg) { if (why) *why = msg; return MADPIPE_EINVAL; };
+    if (!ch || !disc) return bad("null chain or disc");
+    if (ch->L < 1) return bad("L < 1");
+    if (P < 1) return bad("P < 1");
+    if (M <= 0) return bad("M <= 0");
+    if (!(beta > 0.0)) return bad("beta must be > 0 (and not NaN)");
+    if (disc->n_mem < 2 || disc->n_mem > 64) return bad("n_mem outside [2, 64]");
+    if (disc->n_delay < 2 || disc->n_delay > 65535) return bad("n_delay outside [2, 65535]");
+    if (disc->n_periods < 1) return bad("n_periods < 1");
+    if (disc->v_range != 0 && disc->v_range != 1) return bad("v_range not in {0,1}");
+    if (!ch->uF || !ch->uB || !ch->W || !ch->a) return bad("null chain array");
+    if (!host_arrays) return MADPIPE_OK;   // device arrays are checked by the caller
+    const int L = ch->L;
+    double U = 0.0, SC = 0.0;
+    long double sumW = 0, sumA = 0;
+    for (int i = 0; i < L; i++) {
+        const double f = ch->uF[i], b = ch->uB[i];
+        if (!std::isfinite(f) || !std::isfinite(b) || f < 0.0 || b < 0.0 || !(f + b > 0.0))
+            return bad("uF/uB must be finite, >= 0, with uF+uB > 0");
+        if (ch->W[i] < 0) return bad("W < 0");
+        U += f + b;
+        sumW += (long double)ch->W[i];
+    }
+    for (int i = 0; i <= L; i++) {
+        if (ch->a[i] < 0) return bad("a < 0");
+        if (i < L) sumA += (long double)ch->a[i];
+        if (i >= 1 && i <= L - 1) SC += 2.0 * (double)ch->a[i] / beta;
+    }
+    // overflow guards of the int64 memory model: g <= gmax
+    const double lb = U / P;
+    const double vmax = 2.0 * (U + SC) + (U + SC);      // SAFE range at tau = ub (largest)
+    const long double gmax = std::ceil((vmax + U) / lb) + 2.0;
+    const long double worst = 3.0L * sumW + gmax * sumA +
+                              4.0L * (long double)*std::max_element(ch->a, ch->a + L + 1);
+    const long double lim = 9.0e18L;   // < 2^63
+    if (!(worst < lim)) return bad("int64 overflow guard: 3*sum W + g_max*sum a too large");
+    if (!((long double)(M - 1) + (long double)(disc->n_mem - 1) * worst < lim))
+        return bad("int64 overflow guard: (M-1) + (n_mem-1)*memory too large");
+    return MADPIPE_OK;
+}
+
+extern "C" int madpipe_validate(const madpipe_chain *chain, int32_t P, int64_t M, double beta,
+                                const madpipe_disc *disc) {
+    std::string why;
+    int rc = validate_impl(chain, P, M, beta, disc, true, &why);
+    if (rc) g_err = why;
+    return rc;
+}
+
+extern "C" int madpipe_shard(int32_t n_periods, int32_t rank, int32_t world, int32_t *out,
+                             int32_t *count) {
+    if (n_periods < 1 || world < 1 || rank < 0 || rank >= world || !count)
+        return fail(nullptr, MADPIPE_EINVAL, "bad shard arguments");
+    int32_t c = 0;
+    for (int32_t j = rank; j < n_periods; j += world) {
+        if (out) out[c] = j;
+        c++;
+    }
+    *count = c;
+    return MADPIPE_OK;
+}
+
+extern "C" int64_t madpipe_cell_updates(const madpipe_chain *ch, int32_t P,
+                                        const madpipe_disc *disc, double tau) {
+    if (!ch || !disc || ch->L < 1 || P < 1) return -1;
+    if (P < 2) return 0;
+    const int L = ch->L;
+    std::vector<double> Up(L + 1, 0.0);
+    for (int i = 1; i <= L; i++) Up[i] = Up[i - 1] + (ch->uF[i - 1] + ch->uB[i - 1]);
+    int64_t total = 0;
+    int k = 1;
+    for (int l = 1; l <= L; l++) {          // two-pointer scan: kmin(l) is non-decreasing in l
+        if (k > l) k = l;
+        while (k <= l && Up[l] - Up[k - 1] > tau) k++;
+        if (k <= l) total += (int64_t)(l - k + 1);
+    }
+    return total * (int64_t)(P - 1) * disc->n_delay * disc->n_mem;
+}
+
+extern "C" const char *madpipe_last_error(const madpipe_ctx *ctx) {
+    return ctx ? ctx->err.c_str() : g_err.c_str();
+}
+
+// ---------------------------------------------------------------------------
+// context
+// ---------------------------------------------------------------------------
+extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stream,
+                                  int64_t mem_budget) {
+    if (!out) return fail(nullptr, MADPIPE_EINVAL, "null out");
+    *out = nullptr;
+    int n = 0;
+    cudaError_t e = cudaGetDeviceCount(&n);
+    if (e != cudaSuccess || n == 0)
+        return fail(nullptr, MADPIPE_ECUDA, "no CUDA device: %s", cudaGetErrorString(e));
+    if (device < 0 || device >= n) return fail(nullptr, MADPIPE_EINVAL, "bad device %d", device);
+    e = cudaSetDevice(device);
+    if (e != cudaSuccess) return fail(nullptr, MADPIPE_ECUDA, "cudaSetDevice: %s", cudaGetErrorString(e));
+    madpipe_ctx *c = new madpipe_ctx();
+    c->device = device;
+    if (cuda_stream) {
+        c->stream = (cudaStream_t)cuda_stream;
+    } else {
+        if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess) {
+            delete c;
+            return fail(nullptr, MADPIPE_ECUDA, "cudaStreamCreate failed");
+        }
+        c->own_stream = true;
+    }
+    size_t fr = 0, tot = 0;
+    cudaMemGetInfo(&fr, &tot);
+    c->mem_budget = mem_budget > 0 ? mem_budget : (int64_t)(0.6 * (double)fr);
+    cudaEventCreate(&c->ev_a);
+    cudaEventCreate(&c->ev_b);
+    *out = c;
+    return MADPIPE_OK;
+}
+
+extern "C" void madpipe_ctx_destroy(madpipe_ctx *c) {
+    if (!c) return;
+    cudaSetDevice(c->device);
+    cudaStreamSynchronize(c->stream);
+    DevBuf *bufs[] = {&c->tables, &c->jobs, &c->tiles, &c->chains, &c->chain_data, &c->jl,
+                      &c->counts, &c->roots, &c->trace, &c->stages, &c->scratch};
+    for (DevBuf *b : bufs) b->release();
+    for (cudaEvent_t ev : c->ev_pool) cudaEventDestroy(ev);
+    if (c->ev_a) cudaEventDestroy(c->ev_a);
+    if (c->ev_b) cudaEventDestroy(c->ev_b);
+    if (c->own_stream) cudaStreamDestroy(c->stream);
+    delete c;
+}
+
+extern "C" int madpipe_last_timing(const madpipe_ctx *c, double *sweep_ms, double *step_ms,
+                                   int64_t *launches) {
+    if (!c) return MADPIPE_EINVAL;
+    if (sweep_ms) *sweep_ms = c->sweep_ms;
+    if (step_ms) *step_ms = c->step_ms;
+    if (launches) *launches = c->launches;
+    return MADPIPE_OK;
+}
+
+extern "C" int madpipe_last_io(const madpipe_ctx *c, int64_t *h2d_bytes, int64_t *d2h_bytes) {
+    if (!c) return MADPIPE_EINVAL;
+    if (h2d_bytes) *h2d_bytes = c->h2d_bytes;
+    if (d2h_bytes) *d2h_bytes = c->d2h_bytes;
+    return MADPIPE_OK;
+}
+
+extern "C" int madpipe_set_timing(madpipe_ctx *c, int per_launch) {
+    if (!c) return MADPIPE_EINVAL;
+    c->per_launch_timing = per_launch;
+    return MADPIPE_OK;
+}
+
+// ---------------------------------------------------------------------------
+// Engine
+// ---------------------------------------------------------------------------
+namespace {
+
+struct ChainSpec {
+    madpipe_chain c;    // host or device pointers
+    bool on_device;
+    int32_t P;
+    int64_t M;
+    double beta;
+};
+
+struct JobSpec {
+    int chain;
+    int j;
+};
+
+// Upload chains (if on host), allocate derived arrays, run prep_kernel.
+int upload_chains(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, std::vector<ChainDev> &cd) {
+    const int n = (int)cs.size();
+    size_t bytes = 0;
+    auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
+    for (const auto &c : cs) {
+        const size_t L = (size_t)c.c.L;
+        if (!c.on_device) bytes += al(L * 8) * 3 + al((L + 1) * 8);   // uF, uB, W, a
+        bytes += al((L + 1) * 8) * 4 + al(4 * 8);                     // Up, Wp, Ap, C, scal
+    }
+    CUDA_TRY(ctx, ctx->chain_data.ensure(bytes));
+    CUDA_TRY(ctx, ctx->chains.ensure(sizeof(ChainDev) * n));
+    char *base = (char *)ctx->chain_data.p;
+    size_t off = 0;
+    auto take = [&](size_t b) { char *p = base + off; off += al(b); return (void *)p; };
+    cd.resize(n);
+    // host staging of the inputs: one pinned-free contiguous copy per chain
+    for (int i = 0; i < n; i++) {
+        const auto &c = cs[i];
+        const size_t L = (size_t)c.c.L;
+        ChainDev &d = cd[i];
+        if (c.on_device) {
+            d.uF = c.c.uF; d.uB = c.c.uB; d.W = c.c.W; d.a = c.c.a;
+        } else {
+            double *uF = (double *)take(L * 8), *uB = (double *)take(L * 8);
+            int64_t *W = (int64_t *)take(L * 8), *a = (int64_t *)take((L + 1) * 8);
+            CUDA_TRY(ctx, h2d(ctx, uF, c.c.uF, L * 8));
+            CUDA_TRY(ctx, h2d(ctx, uB, c.c.uB, L * 8));
+            CUDA_TRY(ctx, h2d(ctx, W, c.c.W, L * 8));
+            CUDA_TRY(ctx, h2d(ctx, a, c.c.a, (L + 1) * 8));
+            d.uF = uF; d.uB = uB; d.W = W; d.a = a;
+        }
+        d.Up = (double *)take((L + 1) * 8);
+        d.Wp = (int64_t *)take((L + 1) * 8);
+        d.Ap = (int64_t *)take((L + 1) * 8);
+        d.C = (double *)take((L + 1) * 8);
+        d.scal = (double *)take(4 * 8);
+        d.L = c.c.L; d.P = c.P; d.M = c.M; d.beta = c.beta;
+    }
+    CUDA_TRY(ctx, h2d(ctx, ctx->chains.p, cd.data(), sizeof(ChainDev) * n));
+    launch_prep((ChainDev *)ctx->chains.p, n, ctx->stream);
+    ctx->launches++;
+    CUDA_TRY(ctx, cudaGetLastError());
+    return MADPIPE_OK;
+}
+
+size_t table_doubles(const ChainSpec &c, const madpipe_disc *disc) {
+    return (size_t)(c.c.L + 1) * (size_t)disc->n_delay * (size_t)c.P * (size_t)nmp_of(disc->n_mem);
+}
+
+// Tile geometry of one job: np processor rows x vb delay rows.
+void tile_geom(int P, int n_v, int *vb, int *np, int *n_ptiles, int *n_tiles) {
+    const int rows = std::max(1, P - 1);
+    *np = std::min(rows, kThreads);
+    *n_ptiles = (rows + *np - 1) / *np;
+    *vb = std::max(1, std::min(n_v, kThreads / *np));
+    *n_tiles = ((n_v + *vb - 1) / *vb) * *n_ptiles;
+}
+
+struct BatchHook {
+    // called after each batch's tables are complete (before they are reused)
+    virtual int after_batch(madpipe_ctx *ctx, const std::vector<int> &job_ids, Job *jobs_dev) {
+        (void)ctx; (void)job_ids; (void)jobs_dev;
+        return MADPIPE_OK;
+    }
+    virtual ~BatchHook() {}
+};
+
+// Run the DP for a list of jobs in memory-bounded batches.  jl_dev[chain] gets
+// atomicMin'ed with feasible candidate indices; roots_dev (optional) receives
+// each job's root value at its index in `jobs`.  counts_host receives each
+// job's relaxation count.  With early_exit, jobs whose chain already has a
+// smaller feasible candidate are skipped (decided between batches).
+int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vector<ChainDev> &cd,
+             const madpipe_disc *disc, const std::vector<JobSpec> &js, int32_t *jl_dev,
+             double *roots_dev, double *taus_dev, std::vector<uint64_t> *counts_host, bool early_exit,
+             BatchHook *hook, bool timed) {
+    const int nmp = nmp_of(disc->n_mem);
+    const int n_chains = (int)cs.size();
+    if (counts_host) counts_host->assign(js.size(), 0);
+    std::vector<int32_t> jl_host(n_chains, INT32_MAX);
+    size_t next = 0;
+    if (timed) {
+        ctx->sweep_ms = 0.0; ctx->step_ms = 0.0;
+    }
+    std::vector<Job> hjobs;
+    std::vector<int32_t> htiles;
+    std::vector<int> ids;
+    std::vector<unsigned long long> hcounts;
+    const size_t budget = (size_t)ctx->mem_budget;
+    while (next < js.size()) {
+        // ---- form a batch
+        hjobs.clear(); htiles.clear(); ids.clear();
+        size_t used = 0;
+        int maxL = 0;
+        size_t max_slab = 0;
+        for (; next < js.size(); next++) {
+            const JobSpec &s = js[next];
+            if (early_exit && jl_host[s.chain] < s.j) continue;
+            const ChainSpec &c = cs[s.chain];
+            const size_t bytes = table_doubles(c, disc) * 8;
+            if (!hjobs.empty() && used + bytes > budget) break;
+            if (hjobs.empty() && bytes > budget && bytes > ctx->tables.n) {
+                // a single job larger than the budget: try anyway (may fail with ENOMEM)
+            }
+            Job J{};
+            const ChainDev &d = cd[s.chain];
+            J.Up = d.Up; J.Wp = d.Wp; J.Ap = d.Ap; J.a = d.a; J.C = d.C; J.scal = d.scal;
+            J.table = (double *)(uintptr_t)used;   // offset, patched below
+            J.M = c.M; J.L = c.c.L; J.P = c.P; J.n_v = disc->n_delay; J.n_m = disc->n_mem;
+            J.vsafe = disc->v_range == MADPIPE_VRANGE_SAFE; J.j = s.j; J.n_c = disc->n_periods;
+            J.chain = s.chain;
+            J.gid = (int32_t)next;
+            int n_tiles;
+            tile_geom(c.P, disc->n_delay, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
+            J.tile0 = (int32_t)htiles.size();
+            for (int t = 0; t < n_tiles; t++) htiles.push_back((int32_t)hjobs.size());
+            used += (bytes + 255) & ~(size_t)255;
+            maxL = std::max(maxL, J.L);
+            max_slab = std::max(max_slab, (size_t)disc->n_delay * c.P * nmp);
+            hjobs.push_back(J);
+            ids.push_back((int)next);
+        }
+        if (hjobs.empty()) break;
+        CUDA_TRY(ctx, ctx->tables.ensure(used));
+        for (auto &J : hjobs) J.table = (double *)((char *)ctx->tables.p + (uintptr_t)J.table);
+        const int nj = (int)hjobs.size();
+        CUDA_TRY(ctx, ctx->jobs.ensure(sizeof(Job) * nj));
+        CUDA_TRY(ctx, ctx->tiles.ensure(sizeof(int32_t) * htiles.size()));
+        CUDA_TRY(ctx, ctx->counts.ensure(sizeof(unsigned long long) * nj));
+        Job *djobs = (Job *)ctx->jobs.p;
+        CUDA_TRY(ctx, h2d(ctx, djobs, hjobs.data(), sizeof(Job) * nj));
+        CUDA_TRY(ctx, h2d(ctx, ctx->tiles.p, htiles.data(), sizeof(int32_t) * htiles.size()));
+        CUDA_TRY(ctx, cudaMemsetAsync(ctx->counts.p, 0, sizeof(unsigned long long) * nj, ctx->stream));
+        if (timed) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_a, ctx->stream));
+        launch_jobs_init(djobs, nj, ctx->stream);
+        launch_init_slab0(djobs, nj, nmp, (int)std::min(max_slab, (size_t)INT32_MAX), ctx->stream);
+        ctx->launches += 2;
+        const int n_tiles = (int)htiles.size();
+        const bool per_launch = timed && ctx->per_launch_timing;
+        if (per_launch && ctx->ev_pool.size() < (size_t)(2 * maxL)) {
+            while (ctx->ev_pool.size() < (size_t)(2 * maxL)) {
+                cudaEvent_t ev;
+                CUDA_TRY(ctx, cudaEventCreate(&ev));
+                ctx->ev_pool.push_back(ev);
+            }
+        }
+        for (int l = 1; l <= maxL; l++) {
+            if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1)], ctx->stream);
+            launch_step(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, ctx->stream);
+            if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1) + 1], ctx->stream);
+        }
+        ctx->launches += maxL;
+        launch_root(djobs, nj, nmp, jl_dev, roots_dev, taus_dev, ctx->stream);
+        launch_count(djobs, nj, (unsigned long long *)ctx->counts.p, ctx->stream);
+        ctx->launches += 2;
+        CUDA_TRY(ctx, cudaGetLastError());
+        if (timed) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_b, ctx->stream));
+        if (hook) {
+            int rc = hook->after_batch(ctx, ids, djobs);
+            if (rc) return rc;
+        }
+        hcounts.resize(nj);
+        CUDA_TRY(ctx, d2h(ctx, hcounts.data(), ctx->counts.p, sizeof(unsigned long long) * nj));
+        if (early_exit)
+            CUDA_TRY(ctx, d2h(ctx, jl_host.data(), jl_dev, sizeof(int32_t) * n_chains));
+        CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+        if (counts_host)
+            for (int i = 0; i < nj; i++) (*counts_host)[ids[i]] = hcounts[i];
+        if (timed) {
+            float ms = 0.f;
+            cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b);
+            ctx->sweep_ms += ms;
+            if (per_launch) {
+                for (int l = 1; l <= maxL; l++) {
+                    float m2 = 0.f;
+                    cudaEventElapsedTime(&m2, ctx->ev_pool[2 * (l - 1)], ctx->ev_pool[2 * (l - 1) + 1]);
+                    ctx->step_ms += m2;
+                }
+            }
+        }
+    }
+    return MADPIPE_OK;
+}
+
+// Traceback hook: after the winners' tables are built, trace them back.
+struct TraceHook : BatchHook {
+    int nmp, stride;
+    std::vector<TraceOut> outs;
+    std::vector<int32_t> stages;          // [job][3][stride]
+    std::vector<double> taus;
+    int after_batch(madpipe_ctx *ctx, const std::vector<int> &ids, Job *jobs_dev) override {
+        const int nj = (int)ids.size();
+        CUDA_TRY(ctx, ctx->trace.ensure(sizeof(TraceOut) * nj));
+        CUDA_TRY(ctx, ctx->stages.ensure(sizeof(int32_t) * 3 * (size_t)stride * nj));
+        launch_traceback(jobs_dev, nj, nmp, (TraceOut *)ctx->trace.p, (int32_t *)ctx->stages.p,
+                         stride, ctx->stream);
+        ctx->launches++;
+        CUDA_TRY(ctx, cudaGetLastError());
+        std::vector<TraceOut> o(nj);
+        std::vector<int32_t> st(3 * (size_t)stride * nj);
+        std::vector<Job> jb(nj);
+        CUDA_TRY(ctx, d2h(ctx, o.data(), ctx->trace.p, sizeof(TraceOut) * nj));
+        CUDA_TRY(ctx, d2h(ctx, st.data(), ctx->stages.p, sizeof(int32_t) * st.size()));
+        CUDA_TRY(ctx, d2h(ctx, jb.data(), jobs_dev, sizeof(Job) * nj));
+        CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+        for (int i = 0; i < nj; i++) {
+            outs[ids[i]] = o[i];
+            taus[ids[i]] = jb[i].tau;
+            std::copy(st.begin() + (size_t)i * 3 * stride, st.begin() + (size_t)(i + 1) * 3 * stride,
+                      stages.begin() + (size_t)ids[i] * 3 * stride);
+        }
+        return MADPIPE_OK;
+    }
+};
+
+void fill_infeasible(madpipe_alloc *out, int64_t cu) {
+    out->period = INFINITY;
+    out->load_period = INFINITY;
+    out->special_load = INFINITY;
+    out->cand_index = -1;
+    out->n_stages = 0;
+    out->cell_updates = cu;
+}
+
+// Resolve the winners (one job per chain with jstar[c] != INT32_MAX).
+int resolve_impl(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vector<ChainDev> &cd,
+                 const madpipe_disc *disc, const std::vector<int32_t> &jstar, madpipe_alloc *outs) {
+    std::vector<JobSpec> js;
+    int maxL = 1;
+    for (int c = 0; c < (int)cs.size(); c++) {
+        maxL = std::max(maxL, (int)cs[c].c.L);
+        if (jstar[c] != INT32_MAX && jstar[c] >= 0) js.push_back({c, jstar[c]});
+    }
+    TraceHook hook;
+    hook.nmp = nmp_of(disc->n_mem);
+    hook.stride = maxL;
+    hook.outs.assign(js.size(), TraceOut{});
+    hook.stages.assign(js.size() * 3 * (size_t)maxL, 0);
+    hook.taus.assign(js.size(), 0.0);
+    CUDA_TRY(ctx, ctx->jl.ensure(sizeof(int32_t) * std::max<size_t>(1, cs.size())));
+    { int _r = fill_int_max(ctx, (int32_t *)ctx->jl.p, cs.size()); if (_r) return _r; }
+    if (!js.empty()) {
+        int rc = run_jobs(ctx, cs, cd, disc, js, (int32_t *)ctx->jl.p, nullptr, nullptr, nullptr, false,
+                          &hook, false);
+        if (rc) return rc;
+    }
+    for (size_t i = 0; i < js.size(); i++) {
+        madpipe_alloc *o = outs + js[i].chain;
+        const TraceOut &t = hook.outs[i];
+        if (t.status != 0)
+            return fail(ctx, MADPIPE_ESTATE, "resolve of candidate %d: %s", js[i].j,
+                        t.status == 1 ? "root is infeasible" : "traceback found no decision");
+        o->period = hook.taus[i];
+        o->load_period = t.load_period;
+        o->special_load = t.special_load;
+        o->cand_index = js[i].j;
+        o->n_stages = t.n_stages;
+        const int32_t *st = hook.stages.data() + i * 3 * (size_t)maxL;
+        for (int s = 0; s < t.n_stages; s++) {
+            if (o->stage_first) o->stage_first[s] = st[s];
+            if (o->stage_last) o->stage_last[s] = st[maxL + s];
+            if (o->stage_proc) o->stage_proc[s] = st[2 * maxL + s];
+        }
+    }
+    return MADPIPE_OK;
+}
+
+// true if p is device (or managed) memory of the current device
+bool is_device_ptr(const void *p) {
+    cudaPointerAttributes at{};
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+int begin(madpipe_ctx *ctx) {
+    if (!ctx) return fail(nullptr, MADPIPE_EINVAL, "null ctx");
+    ctx->err.clear();
+    ctx->launches = 0;
+    ctx->h2d_bytes = 0;
+    ctx->d2h_bytes = 0;
+    cudaError_t e = cudaSetDevice(ctx->device);
+    if (e != cudaSuccess) return fail(ctx, MADPIPE_ECUDA, "cudaSetDevice: %s", cudaGetErrorString(e));
+    return MADPIPE_OK;
+}
+
+int check_one(madpipe_ctx *ctx, const madpipe_chain *ch, int32_t P, int64_t M, double beta,
+              const madpipe_disc *disc, bool host) {
+    std::string why;
+    int rc = validate_impl(ch, P, M, beta, disc, host, &why);
+    if (rc) return fail(ctx, rc, "invalid argument: %s", why.c_str());
+    return MADPIPE_OK;
+}
+
+std::vector<JobSpec> shard_jobs(int chain, int n_c, int rank, int world) {
+    std::vector<JobSpec> js;
+    for (int j = rank; j < n_c; j += world) js.push_back({chain, j});
+    return js;
+}
+
+int solve_common(madpipe_ctx *ctx, const madpipe_chain *chain, bool on_device, int32_t P, int64_t M,
+                 double beta, const madpipe_disc *disc, madpipe_alloc *out) {
+    int rc = begin(ctx);
+    if (rc) return rc;
+    if (!out) return fail(ctx, MADPIPE_EINVAL, "null out");
+    rc = check_one(ctx, chain, P, M, beta, disc, !on_device);
+    if (rc) return rc;
+    std::vector<ChainSpec> cs{{*chain, on_device, P, M, beta}};
+    std::vector<ChainDev> cd;
+    rc = upload_chains(ctx, cs, cd);
+    if (rc) return rc;
+    CUDA_TRY(ctx, ctx->jl.ensure(sizeof(int32_t)));
+    { int _r = fill_int_max(ctx, (int32_t *)ctx->jl.p, 1); if (_r) return _r; }
+    std::vector<uint64_t> counts;
+    rc = run_jobs(ctx, cs, cd, disc, shard_jobs(0, disc->n_periods, 0, 1), (int32_t *)ctx->jl.p,
+                  nullptr, nullptr, &counts, disc->early_exit != 0, nullptr, true);
+    if (rc) return rc;
+    int64_t cu = 0;
+    for (auto x : counts) cu += (int64_t)x;
+    int32_t jstar = INT32_MAX;
+    CUDA_TRY(ctx, d2h(ctx, &jstar, ctx->jl.p, sizeof(int32_t)));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    if (jstar == INT32_MAX) {
+        fill_infeasible(out, cu);
+        return MADPIPE_INFEASIBLE;
+    }
+    std::vector<int32_t> js{jstar};
+    rc = resolve_impl(ctx, cs, cd, disc, js, out);
+    out->cell_updates = cu;
+    return rc;
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------------------
+// public entry points
+// ---------------------------------------------------------------------------
+extern "C" int madpipe_solve(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                             double beta, const madpipe_disc *disc, madpipe_alloc *out) {
+    return solve_common(ctx, chain, false, P, M, beta, disc, out);
+}
+
+extern "C" int madpipe_solve_dev(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                                 double beta, const madpipe_disc *disc, madpipe_alloc *out) {
+    return solve_common(ctx, chain, true, P, M, beta, disc, out);
+}
+
+extern "C" int madpipe_sweep(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                             double beta, const madpipe_disc *disc, int32_t rank, int32_t world,
+                             int32_t *j_local, int64_t *cell_updates_out) {
+    int rc = begin(ctx);
+    if (rc) return rc;
+    if (world < 1 || rank < 0 || rank >= world || !j_local)
+        return fail(ctx, MADPIPE_EINVAL, "bad rank/world/j_local");
+    const bool dev = chain && is_device_ptr(chain->uF);
+    rc = check_one(ctx, chain, P, M, beta, disc, !dev);
+    if (rc) return rc;
+    std::vector<ChainSpec> cs{{*chain, dev, P, M, beta}};
+    std::vector<ChainDev> cd;
+    rc = upload_chains(ctx, cs, cd);
+    if (rc) return rc;
+    { int _r = fill_int_max(ctx, (int32_t *)j_local, 1); if (_r) return _r; }
+    std::vector<uint64_t> counts;
+    rc = run_jobs(ctx, cs, cd, disc, shard_jobs(0, disc->n_periods, rank, world), j_local, nullptr,
+                  nullptr, &counts, disc->early_exit != 0, nullptr, true);
+    if (rc) return rc;
+    int64_t cu = 0;
+    for (auto x : counts) cu += (int64_t)x;
+    if (cell_updates_out) *cell_updates_out = cu;
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    return MADPIPE_OK;
+}
+
+extern "C" int madpipe_resolve(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                               double beta, const madpipe_disc *disc, const int32_t *j_star,
+                               madpipe_alloc *out) {
+    int rc = begin(ctx);
+    if (rc) return rc;
+    if (!j_star || !out) return fail(ctx, MADPIPE_EINVAL, "null j_star/out");
+    const bool dev = chain && is_device_ptr(chain->uF);
+    rc = check_one(ctx, chain, P, M, beta, disc, !dev);
+    if (rc) return rc;
+    int32_t js = INT32_MAX;
+    CUDA_TRY(ctx, d2h(ctx, &js, j_star, sizeof(int32_t)));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    if (js == INT32_MAX) {
+        fill_infeasible(out, 0);
+        return MADPIPE_INFEASIBLE;
+    }
+    if (js < 0 || js >= disc->n_periods) return fail(ctx, MADPIPE_EINVAL, "j_star out of range");
+    std::vector<ChainSpec> cs{{*chain, dev, P, M, beta}};
+    std::vector<ChainDev> cd;
+    rc = upload_chains(ctx, cs, cd);
+    if (rc) return rc;
+    std::vector<int32_t> jv{js};
+    int64_t keep = out->cell_updates;
+    rc = resolve_impl(ctx, cs, cd, disc, jv, out);
+    out->cell_updates = keep;
+    return rc;
+}
+
+extern "C" int madpipe_solve_batch(madpipe_ctx *ctx, int32_t n, const madpipe_chain *chains,
+                                   const int32_t *P, const int64_t *M, const double *beta,
+                                   const madpipe_disc *disc, madpipe_alloc *out) {
+    int rc = begin(ctx);
+    if (rc) return rc;
+    if (n < 1 || !chains || !P || !M || !beta || !out)
+        return fail(ctx, MADPIPE_EINVAL, "bad batch arguments");
+    std::vector<ChainSpec> cs;
+    for (int i = 0; i < n; i++) {
+        rc = check_one(ctx, &chains[i], P[i], M[i], beta[i], disc, true);
+        if (rc) return fail(ctx, rc, "chain %d: %s", i, ctx->err.c_str());
+        cs.push_back({chains[i], false, P[i], M[i], beta[i]});
+    }
+    std::vector<ChainDev> cd;
+    rc = upload_chains(ctx, cs, cd);
+    if (rc) return rc;
+    CUDA_TRY(ctx, ctx->jl.ensure(sizeof(int32_t) * n));
+    { int _r = fill_int_max(ctx, (int32_t *)ctx->jl.p, n); if (_r) return _r; }
+    // candidate-major order keeps small (cheap) periods of every chain first,
+    // so early exit prunes the expensive large periods
+    std::vector<JobSpec> js;
+    for (int j = 0; j < disc->n_periods; j++)
+        for (int c = 0; c < n; c++) js.push_back({c, j});
+    std::vector<uint64_t> counts;
+    rc = run_jobs(ctx, cs, cd, disc, js, (int32_t *)ctx->jl.p, nullptr, nullptr, &counts,
+                  disc->early_exit != 0, nullptr, true);
+    if (rc) return rc;
+    std::vector<int64_t> cu(n, 0);
+    for (size_t i = 0; i < js.size(); i++) cu[js[i].chain] += (int64_t)counts[i];
+    std::vector<int32_t> jstar(n);
+    CUDA_TRY(ctx, d2h(ctx, jstar.data(), ctx->jl.p, sizeof(int32_t) * n));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    for (int i = 0; i < n; i++) fill_infeasible(&out[i], cu[i]);
+    rc = resolve_impl(ctx, cs, cd, disc, jstar, out);
+    for (int i = 0; i < n; i++) out[i].cell_updates = cu[i];
+    return rc;
+}
+
+extern "C" int madpipe_candidates(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                                  double beta, const madpipe_disc *disc, double *tau_out,
+                                  double *root_out) {
+    int rc = begin(ctx);
+    if (rc) return rc;
+    rc = check_one(ctx, chain, P, M, beta, disc, true);
+    if (rc) return rc;
+    std::vector<ChainSpec> cs{{*chain, false, P, M, beta}};
+    std::vector<ChainDev> cd;
+    rc = upload_chains(ctx, cs, cd);
+    if (rc) return rc;
+    const int n_c = disc->n_periods;
+    CUDA_TRY(ctx, ctx->jl.ensure(sizeof(int32_t)));
+    { int _r = fill_int_max(ctx, (int32_t *)ctx->jl.p, 1); if (_r) return _r; }
+    CUDA_TRY(ctx, ctx->scratch.ensure(sizeof(double) * 2 * n_c));
+    double *roots_dev = (double *)ctx->scratch.p, *taus_dev = roots_dev + n_c;
+    madpipe_disc d2 = *disc;
+    d2.early_exit = 0;
+    std::vector<JobSpec> js = shard_jobs(0, n_c, 0, 1);
+    rc = run_jobs(ctx, cs, cd, &d2, js, (int32_t *)ctx->jl.p, roots_dev, taus_dev, nullptr, false,
+                  nullptr, true);
+    if (rc) return rc;
+    if (root_out)
+        CUDA_TRY(ctx, d2h(ctx, root_out, roots_dev, sizeof(double) * n_c));
+    if (tau_out)
+        CUDA_TRY(ctx, d2h(ctx, tau_out, taus_dev, sizeof(double) * n_c));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    return MADPIPE_OK;
+}
+
+namespace {
+struct ExportHook : BatchHook {
+    int nmp, L, P, n_v, n_m;
+    double *A_dev = nullptr;
+    int32_t *arg_dev = nullptr;
+    int after_batch(madpipe_ctx *ctx, const std::vector<int> &, Job *jobs_dev) override {
+        launch_export(jobs_dev, nmp, A_dev, L, P, n_v, n_m, ctx->stream);
+        ctx->launches++;
+        if (arg_dev) { launch_argmin(jobs_dev, nmp, arg_dev, L, P, n_v, n_m, ctx->stream); ctx->launches++; }
+        CUDA_TRY(ctx, cudaGetLastError());
+        return MADPIPE_OK;
+    }
+};
+}  // namespace
+
+extern "C" int madpipe_dp_table(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                                double beta, const madpipe_disc *disc, int32_t j, double *A_out,
+                                int32_t *arg_out) {
+    int rc = begin(ctx);
+    if (rc) return rc;
+    rc = check_one(ctx, chain, P, M, beta, disc, true);
+    if (rc) return rc;
+    if (j < 0 || j >= disc->n_periods || !A_out) return fail(ctx, MADPIPE_EINVAL, "bad j / A_out");
+    std::vector<ChainSpec> cs{{*chain, false, P, M, beta}};
+    std::vector<ChainDev> cd;
+    rc = upload_chains(ctx, cs, cd);
+    if (rc) return rc;
+    const size_t cells = (size_t)(chain->L + 1) * P * disc->n_delay * disc->n_mem;
+    CUDA_TRY(ctx, ctx->scratch.ensure(cells * (sizeof(double) + sizeof(int32_t))));
+    ExportHook hook;
+    hook.nmp = nmp_of(disc->n_mem); hook.L = chain->L; hook.P = P; hook.n_v = disc->n_delay;
+    hook.n_m = disc->n_mem;
+    hook.A_dev = (double *)ctx->scratch.p;
+    hook.arg_dev = arg_out ? (int32_t *)((char *)ctx->scratch.p + cells * sizeof(double)) : nullptr;
+    CUDA_TRY(ctx, ctx->jl.ensure(sizeof(int32_t)));
+    { int _r = fill_int_max(ctx, (int32_t *)ctx->jl.p, 1); if (_r) return _r; }
+    std::vector<JobSpec> js{{0, j}};
+    rc = run_jobs(ctx, cs, cd, disc, js, (int32_t *)ctx->jl.p, nullptr, nullptr, nullptr, false, &hook,
+                  false);
+    if (rc) return rc;
+    CUDA_TRY(ctx, d2h(ctx, A_out, hook.A_dev, cells * sizeof(double)));
+    if (arg_out)
+        CUDA_TRY(ctx, d2h(ctx, arg_out, hook.arg_dev, cells * sizeof(int32_t)));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    return MADPIPE_OK;
+}

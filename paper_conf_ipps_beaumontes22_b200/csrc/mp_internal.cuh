@@ -1,0 +1,82 @@
+// mp_internal.cuh -- internal structures of libmadpipe (B200 / sm_100a).
+//
+// Product code: shares nothing with oracle/ (the CPU oracle used by tests).
+// Paper references: "P:n" = line n of the MadPipe paper text; "Qn" = the
+// readings listed in DESIGN.md section 3.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace mp {
+
+// Per-chain device arrays (section 8(a) step a1, P:155 / P:159 / P:147).
+struct ChainDev {
+    const double  *uF, *uB;     // [L]
+    const int64_t *W, *a;       // [L], [L+1]
+    double  *Up;                // [L+1] prefix sums of uF+uB
+    int64_t *Wp, *Ap;           // [L+1] prefix sums of W_i and a_{i-1}
+    double  *C;                 // [L+1] C[i] = 2 a_i / beta (i=1..L-1), C[0]=C[L]=0
+    double  *scal;              // [4]  SC, lb, ub, U(1,L)
+    int32_t L, P;
+    int64_t M;
+    double  beta;
+};
+
+// One unit of the sweep: a (chain, candidate period) pair.
+struct Job {
+    const double  *Up;
+    const int64_t *Wp, *Ap, *a;
+    const double  *C;
+    double  *table;     // [(L+1)][n_v][P][NMP] fp64, m innermost
+    double   tau, dV;   // filled on device by jobs_init_kernel
+    int64_t  M;
+    int32_t  L, P, n_v, n_m;
+    int32_t  vsafe;     // 1 = SAFE v_range (saturate), 0 = PAPER (overflow infeasible)
+    int32_t  j;         // candidate index
+    int32_t  n_c;       // number of candidates of the chain
+    int32_t  chain;     // chain index (batch API)
+    int32_t  tile0;     // first tile of this job in the step grid
+    int32_t  vb;        // delay rows per tile
+    int32_t  np;        // p rows (>=1) per tile
+    int32_t  n_ptiles;  // tiles along p
+    int32_t  gid;       // index of the job in the caller's job list (root/tau export)
+    const double *scal; // chain scalars (SC, lb, ub, U(1,L))
+};
+
+// Result of a traceback, written by traceback_kernel.
+struct TraceOut {
+    double  load_period;
+    double  special_load;
+    int32_t n_stages;
+    int32_t status;     // 0 ok, 1 infeasible root, 2 broken path
+    // followed in memory by stage arrays (first,last,proc) of capacity L each
+};
+
+constexpr int kThreads = 256;        // threads per step CTA
+constexpr int kTransSmem = 2048;     // transition entries staged per chunk
+constexpr int kMaxKChunk = 512;
+
+// Transition packing (int32): bit 31 set = skip this k;
+//   bits 0..15 vn, bits 16..23 d (clamped to 255), bit 24 nf.
+__host__ __device__ inline int32_t pack_trans(int vn, int64_t d, bool nf) {
+    int dd = d > 255 ? 255 : (int)d;
+    return (int32_t)((unsigned)vn | ((unsigned)dd << 16) | ((nf ? 1u : 0u) << 24));
+}
+
+// kernel launchers (mp_kernels.cu)
+void launch_prep(ChainDev *chains_dev, int n_chains, cudaStream_t s);
+void launch_jobs_init(Job *jobs, int n_jobs, cudaStream_t s);
+void launch_init_slab0(const Job *jobs, int n_jobs, int nmp, int max_cells, cudaStream_t s);
+void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp,
+                 cudaStream_t s);
+void launch_root(const Job *jobs, int n_jobs, int nmp, int32_t *jl_per_chain, double *root_out,
+                 double *tau_out, cudaStream_t s);
+void launch_count(const Job *jobs, int n_jobs, unsigned long long *counts, cudaStream_t s);
+void launch_traceback(const Job *jobs, int n_jobs, int nmp, TraceOut *outs, int32_t *stages,
+                      int stage_stride, cudaStream_t s);
+void launch_argmin(const Job *job, int nmp, int32_t *arg_out, int L, int P, int n_v, int n_m,
+                   cudaStream_t s);
+void launch_export(const Job *job, int nmp, double *A_out, int L, int P, int n_v, int n_m,
+                   cudaStream_t s);
+
+}  // namespace mp

@@ -1,0 +1,189 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, on the same
+seeded inputs.  Bar (BASELINE.json north_star): bit-exact fp64 DP values, decisions,
+candidate periods and allocations; the 1F1B* simulator verifies every returned
+allocation (period within 1e-12 relative, memory <= M)."""
+import math
+
+import numpy as np
+import pytest
+
+import chaingen
+import oracle
+import paper_conf_ipps_beaumontes22_b200 as mp
+from oracle import simulator
+from paper_conf_ipps_beaumontes22_b200 import configs
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    import torch
+    assert torch.cuda.is_available()
+    c = mp.Context(0)
+    yield c
+    c.close()
+
+
+def _args(cfg):
+    return (cfg["P"], cfg["M"], cfg["beta"], cfg["n_mem"], cfg["n_delay"], cfg["n_periods"])
+
+
+def _same_solution(got, ref):
+    for key in ("rc", "cand_index", "period", "special_load", "load_period", "stages"):
+        assert got[key] == ref[key], (key, got[key], ref[key])
+
+
+def _verify(ch, P, M, beta, res):
+    if res["rc"] != 0:
+        return
+    rep = simulator.check_allocation(ch, P, M, beta, res["period"], res["stages"],
+                                     res["load_period"], res["special_load"])
+    assert rep["errors"] == [], rep["errors"]
+
+
+# ---------------------------------------------------------------- toy: everything, every candidate
+def test_toy_full_tables_every_candidate(ctx):
+    cfg = configs.load("toy")
+    ch = chaingen.make(cfg["chain"])
+    a = _args(cfg)
+    ref = oracle.solve(ch, *a)
+    tau, root = ctx.candidates(ch, *a)
+    assert np.array_equal(tau, ref["tau"]) and np.array_equal(root, ref["root"])
+    for j in range(cfg["n_periods"]):
+        A, ARG = ctx.dp_table(ch, *a, j=j)
+        A_ref, ARG_ref, _ = oracle.table(ch, cfg["P"], cfg["M"], cfg["beta"], cfg["n_mem"],
+                                         cfg["n_delay"], 0, ref["tau"][j])
+        assert np.array_equal(A, A_ref), j
+        assert np.array_equal(ARG, ARG_ref), j
+    got = ctx.solve(ch, *a)
+    _same_solution(got, ref)
+    assert got["cell_updates"] == ref["cell_updates"]
+    _verify(ch, cfg["P"], cfg["M"], cfg["beta"], got)
+
+
+# ---------------------------------------------------------------- fuzz: tiny chains, all features
+def _fuzz_cases(n, seed):
+    rng = np.random.default_rng(seed)
+    for i in range(n):
+        L = int(rng.integers(1, 14))
+        P = int(rng.integers(1, 7))
+        ch = chaingen.tiny(rng, L, integer_times=bool(i % 3 == 0), zero_mem=bool(i % 7 == 0))
+        n_m = int(rng.choice([2, 3, 4, 8, 11, 16, 33]))
+        n_v = int(rng.choice([2, 5, 16, 51, 100]))
+        n_c = int(rng.choice([1, 3, 17]))
+        vr = int(rng.integers(0, 2))
+        mem = 3 * int(ch["W"].sum()) + 3 * int(ch["a"].sum()) + 1
+        M = int(mem * rng.uniform(0.1, 1.0)) + 1
+        beta = float(rng.choice([math.inf, rng.uniform(5.0, 60.0)]))
+        yield ch, P, M, beta, n_m, n_v, n_c, vr
+
+
+def test_fuzz_roots_tables_solutions(ctx):
+    for ch, P, M, beta, n_m, n_v, n_c, vr in _fuzz_cases(120, 7):
+        ref = oracle.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
+        tau, root = ctx.candidates(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
+        assert np.array_equal(tau, ref["tau"])
+        assert np.array_equal(root, ref["root"]), (P, n_m, n_v, vr)
+        got = ctx.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
+        _same_solution(got, ref)
+        assert got["cell_updates"] == ref["cell_updates"]
+        j = max(ref["cand_index"], 0)
+        A, ARG = ctx.dp_table(ch, P, M, beta, n_m, n_v, n_c, j=j, v_range=vr)
+        A_ref, ARG_ref, _ = oracle.table(ch, P, M, beta, n_m, n_v, vr, ref["tau"][j])
+        assert np.array_equal(A, A_ref) and np.array_equal(ARG, ARG_ref)
+        _verify(ch, P, M, beta, got)
+
+
+def test_early_exit_same_answer(ctx):
+    for ch, P, M, beta, n_m, n_v, n_c, vr in _fuzz_cases(30, 8):
+        full = ctx.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
+        ee = ctx.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr, early_exit=True)
+        _same_solution(ee, full)
+        assert ee["cell_updates"] <= full["cell_updates"]
+
+
+def test_paper_discretisation(ctx):
+    """The paper's own grid: 11 memory levels, 51 delay levels."""
+    ch = chaingen.resnet50()
+    a = (4, 8 * 10**9, 12e9, 11, 51, 16)
+    ref = oracle.solve(ch, *a, n_threads=8)
+    got = ctx.solve(ch, *a)
+    _same_solution(got, ref)
+    tau, root = ctx.candidates(ch, *a)
+    assert np.array_equal(root, ref["root"])
+
+
+# ---------------------------------------------------------------- BASELINE configs
+def _sampled(ref_tau, jstar, n_c, extra_hi=4):
+    js = set(range(0, min(jstar + 3, n_c)))
+    hi = np.linspace(jstar + 3, n_c - 1, extra_hi).astype(int) if jstar + 3 < n_c else []
+    js.update(int(x) for x in hi)
+    return sorted(js)
+
+
+@pytest.mark.parametrize("name", ["resnet50", "inception_v3", "vgg19"])
+def test_cnn_configs(ctx, name):
+    cfg = configs.load(name)
+    ch = chaingen.make(cfg["chain"])
+    assert chaingen.digest(ch) == cfg["digest"]
+    a = _args(cfg)
+    got = ctx.solve(ch, *a)
+    assert got["cand_index"] == cfg["oracle_cand_index"]
+    ref = oracle.solve(ch, *a, early_exit=True, n_threads=8)
+    _same_solution(got, ref)
+    tau, root = ctx.candidates(ch, *a)
+    assert np.array_equal(tau, ref["tau"])
+    for j in _sampled(ref["tau"], ref["cand_index"], cfg["n_periods"]):
+        A_ref, _, _ = oracle.table(ch, cfg["P"], cfg["M"], cfg["beta"], cfg["n_mem"],
+                                   cfg["n_delay"], 0, tau[j], with_arg=False)
+        assert root[j] == A_ref[-1, cfg["P"] - 1, 0, 0], j
+    # full table and decisions of the winner
+    j = got["cand_index"]
+    A, ARG = ctx.dp_table(ch, *a, j=j)
+    A_ref, ARG_ref, _ = oracle.table(ch, cfg["P"], cfg["M"], cfg["beta"], cfg["n_mem"],
+                                     cfg["n_delay"], 0, tau[j])
+    assert np.array_equal(A, A_ref) and np.array_equal(ARG, ARG_ref)
+    _verify(ch, cfg["P"], cfg["M"], cfg["beta"], got)
+
+
+def test_gpt_config_sampled(ctx):
+    """Full BASELINE size, bench launch configuration: the solve, the winner and a
+    sample of candidate roots (cheap low periods + stratified high ones)."""
+    cfg = configs.load("gpt")
+    ch = chaingen.make(cfg["chain"])
+    assert chaingen.digest(ch) == cfg["digest"]
+    a = _args(cfg)
+    got = ctx.solve(ch, *a)
+    assert got["cand_index"] == cfg["oracle_cand_index"]
+    ref = oracle.solve(ch, *a, early_exit=True, n_threads=8)
+    _same_solution(got, ref)
+    _verify(ch, cfg["P"], cfg["M"], cfg["beta"], got)
+    ee = ctx.solve(ch, *a, early_exit=True)
+    _same_solution(ee, ref)
+    tau, root = ctx.candidates(ch, *a)
+    assert np.array_equal(tau, ref["tau"])
+    jstar = ref["cand_index"]
+    for j in [0, max(0, jstar - 1), jstar, min(jstar + 1, 1023), 300]:
+        A_ref, _, _ = oracle.table(ch, cfg["P"], cfg["M"], cfg["beta"], cfg["n_mem"],
+                                   cfg["n_delay"], 0, tau[j], with_arg=False)
+        assert root[j] == A_ref[-1, cfg["P"] - 1, 0, 0], j
+
+
+def test_batch_config_sampled(ctx):
+    cfg = configs.load("batch")
+    rng = np.random.default_rng(0)
+    pick = sorted(rng.choice(len(cfg["chains"]), size=24, replace=False).tolist())
+    chains, Ps, Ms, Bs = [], [], [], []
+    for i in pick:
+        c = cfg["chains"][i]
+        ch = chaingen.random_chain(c["seed"])
+        assert chaingen.digest(ch) == c["digest"]
+        chains.append(ch); Ps.append(c["P"]); Ms.append(c["M"]); Bs.append(c["beta"])
+    res = ctx.solve_batch(chains, Ps, Ms, Bs, cfg["n_mem"], cfg["n_delay"], cfg["n_periods"])
+    for i, ch, P, M, B, got in zip(pick, chains, Ps, Ms, Bs, res):
+        ref = oracle.solve(ch, P, M, B, cfg["n_mem"], cfg["n_delay"], cfg["n_periods"],
+                           early_exit=True, n_threads=8)
+        _same_solution(got, ref)
+        assert got["cand_index"] == cfg["chains"][i]["oracle_cand_index"]
+        _verify(ch, P, M, B, got)
