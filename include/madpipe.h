@@ -177,6 +177,12 @@ int madpipe_set_timing(madpipe_ctx *ctx, int per_launch);
 /* Bytes the last call copied host->device and device->host (inputs, job
  * descriptors, results); for the bench's end-to-end record. */
 int madpipe_last_io(const madpipe_ctx *ctx, int64_t *h2d_bytes, int64_t *d2h_bytes);
+/* Relaxation counts of the last sweep: cell_updates as in madpipe_alloc (every
+ * (k, l, v, p, m) of the windows) and effective_updates, the
+ * relaxations whose transition is live (not skipped by a delay overflow, a
+ * communication longer than the period, or neither N nor S fitting) -- the
+ * ones that read the DP table. */
+int madpipe_last_counts(const madpipe_ctx *ctx, int64_t *cell_updates, int64_t *effective_updates);
 
 #ifdef __cplusplus
 }

@@ -182,6 +182,11 @@ class Context:
         N.check(self._lib.madpipe_last_io(self.h, ctypes.byref(a), ctypes.byref(b)))
         return dict(h2d_bytes=a.value, d2h_bytes=b.value)
 
+    def last_counts(self):
+        a = ctypes.c_int64(); b = ctypes.c_int64()
+        N.check(self._lib.madpipe_last_counts(self.h, ctypes.byref(a), ctypes.byref(b)))
+        return dict(cell_updates=a.value, effective_updates=b.value)
+
     def last_timing(self):
         s = ctypes.c_double(); k = ctypes.c_double(); n = ctypes.c_int64()
         N.check(self._lib.madpipe_last_timing(self.h, ctypes.byref(s), ctypes.byref(k), ctypes.byref(n)))

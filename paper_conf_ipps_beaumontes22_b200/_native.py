@@ -74,6 +74,7 @@ def lib():
         "madpipe_last_timing": (ctypes.c_int, [vp, _dp, _dp, _i64p]),
         "madpipe_set_timing": (ctypes.c_int, [vp, ctypes.c_int]),
         "madpipe_last_io": (ctypes.c_int, [vp, _i64p, _i64p]),
+        "madpipe_last_counts": (ctypes.c_int, [vp, _i64p, _i64p]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -86,7 +87,8 @@ def lib():
 EXPORTED = ["madpipe_ctx_create", "madpipe_ctx_destroy", "madpipe_last_error", "madpipe_validate",
             "madpipe_shard", "madpipe_cell_updates", "madpipe_solve", "madpipe_solve_dev",
             "madpipe_sweep", "madpipe_resolve", "madpipe_solve_batch", "madpipe_candidates",
-            "madpipe_dp_table", "madpipe_last_timing", "madpipe_set_timing", "madpipe_last_io"]
+            "madpipe_dp_table", "madpipe_last_timing", "madpipe_set_timing", "madpipe_last_io",
+            "madpipe_last_counts"]
 
 
 class MadpipeError(RuntimeError):

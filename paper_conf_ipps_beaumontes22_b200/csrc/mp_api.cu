@@ -47,6 +47,7 @@ struct madpipe_ctx {
     double sweep_ms = 0.0, step_ms = 0.0;
     int64_t launches = 0;
     int64_t h2d_bytes = 0, d2h_bytes = 0;
+    int64_t last_cell_updates = 0, last_effective = 0;
     int per_launch_timing = 0;
     std::vector<cudaEvent_t> ev_pool;
 };
@@ -241,6 +242,14 @@ extern "C" int madpipe_last_timing(const madpipe_ctx *c, double *sweep_ms, doubl
     return MADPIPE_OK;
 }
 
+extern "C" int madpipe_last_counts(const madpipe_ctx *c, int64_t *cell_updates,
+                                   int64_t *effective_updates) {
+    if (!c) return MADPIPE_EINVAL;
+    if (cell_updates) *cell_updates = c->last_cell_updates;
+    if (effective_updates) *effective_updates = c->last_effective;
+    return MADPIPE_OK;
+}
+
 extern "C" int madpipe_last_io(const madpipe_ctx *c, int64_t *h2d_bytes, int64_t *d2h_bytes) {
     if (!c) return MADPIPE_EINVAL;
     if (h2d_bytes) *h2d_bytes = c->h2d_bytes;
@@ -356,6 +365,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
     size_t next = 0;
     if (timed) {
         ctx->sweep_ms = 0.0; ctx->step_ms = 0.0;
+        ctx->last_cell_updates = 0; ctx->last_effective = 0;
     }
     std::vector<Job> hjobs;
     std::vector<int32_t> htiles;
@@ -401,11 +411,12 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         const int nj = (int)hjobs.size();
         CUDA_TRY(ctx, ctx->jobs.ensure(sizeof(Job) * nj));
         CUDA_TRY(ctx, ctx->tiles.ensure(sizeof(int32_t) * htiles.size()));
-        CUDA_TRY(ctx, ctx->counts.ensure(sizeof(unsigned long long) * nj));
+        CUDA_TRY(ctx, ctx->counts.ensure(sizeof(unsigned long long) * 2 * nj));
+        for (int i = 0; i < nj; i++) hjobs[i].eff = (unsigned long long *)ctx->counts.p + nj + i;
         Job *djobs = (Job *)ctx->jobs.p;
         CUDA_TRY(ctx, h2d(ctx, djobs, hjobs.data(), sizeof(Job) * nj));
         CUDA_TRY(ctx, h2d(ctx, ctx->tiles.p, htiles.data(), sizeof(int32_t) * htiles.size()));
-        CUDA_TRY(ctx, cudaMemsetAsync(ctx->counts.p, 0, sizeof(unsigned long long) * nj, ctx->stream));
+        CUDA_TRY(ctx, cudaMemsetAsync(ctx->counts.p, 0, sizeof(unsigned long long) * 2 * nj, ctx->stream));
         if (timed) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_a, ctx->stream));
         launch_jobs_init(djobs, nj, ctx->stream);
         launch_init_slab0(djobs, nj, nmp, (int)std::min(max_slab, (size_t)INT32_MAX), ctx->stream);
@@ -434,13 +445,19 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             int rc = hook->after_batch(ctx, ids, djobs);
             if (rc) return rc;
         }
-        hcounts.resize(nj);
-        CUDA_TRY(ctx, d2h(ctx, hcounts.data(), ctx->counts.p, sizeof(unsigned long long) * nj));
+        hcounts.resize(2 * nj);
+        CUDA_TRY(ctx, d2h(ctx, hcounts.data(), ctx->counts.p, sizeof(unsigned long long) * 2 * nj));
         if (early_exit)
             CUDA_TRY(ctx, d2h(ctx, jl_host.data(), jl_dev, sizeof(int32_t) * n_chains));
         CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
         if (counts_host)
             for (int i = 0; i < nj; i++) (*counts_host)[ids[i]] = hcounts[i];
+        if (timed) {
+            for (int i = 0; i < nj; i++) {
+                ctx->last_cell_updates += (int64_t)hcounts[i];
+                ctx->last_effective += (int64_t)hcounts[nj + i];
+            }
+        }
         if (timed) {
             float ms = 0.f;
             cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b);

@@ -41,6 +41,7 @@ struct Job {
     int32_t  n_ptiles;  // tiles along p
     int32_t  gid;       // index of the job in the caller's job list (root/tau export)
     const double *scal; // chain scalars (SC, lb, ub, U(1,L))
+    unsigned long long *eff;  // effective (non-skipped) relaxations of this job
 };
 
 // Result of a traceback, written by traceback_kernel.

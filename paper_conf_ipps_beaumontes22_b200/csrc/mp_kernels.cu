@@ -245,12 +245,21 @@ __global__ void __launch_bounds__(kThreads) step_kernel(const Job *__restrict__ 
     for (int kc0 = kmin; kc0 <= l; kc0 += kc_len) {
         const int nk = min(kc_len, l + 1 - kc0);
         __syncthreads();
+        unsigned live = 0;
         for (int e = tid; e < nk * vcount; e += kThreads) {
             const int kk = e / vcount, v2 = e - kk * vcount;
             const int k = kc0 + kk;
             const double Ukl = __dsub_rn(Ul, J.Up[k - 1]);
-            s_tr[e] = transition(J, k, l, v0 + v2, Ukl, nullptr);
+            const int32_t tr = transition(J, k, l, v0 + v2, Ukl, nullptr);
+            s_tr[e] = tr;
+            live += tr >= 0;
             if (v2 == 0) s_U[kk] = Ukl;
+        }
+        if (pt == 0) {   // count each live (k, l, v) once: it feeds (P-1) n_m relaxations
+            for (int o = 16; o > 0; o >>= 1) live += __shfl_xor_sync(0xffffffffu, live, o);
+            if ((tid & 31) == 0 && live)
+                atomicAdd(J.eff, (unsigned long long)live * (unsigned long long)(J.P - 1) *
+                                     (unsigned long long)n_m);
         }
         __syncthreads();
         if (!active) continue;
