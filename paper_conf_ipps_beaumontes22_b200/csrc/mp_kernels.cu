@@ -162,6 +162,21 @@ __device__ __forceinline__ int kmin_of(const Job &J, int l) {
     return lo;
 }
 
+// Smallest k in [1,l] whose weights alone fit: 3 (Wp[l] - Wp[k-1]) <= M; l+1 if
+// none.  For k below it, M(k,l,g) >= 3 sum W > M for every g >= 0, so neither a
+// normal GPU nor the special one (M(k,l,g-1) with g >= 1) can
+// take stage k..l: transition() would return kSkip.  Pruning these k is exact.
+__device__ __forceinline__ int kmin_mem(const Job &J, int l) {
+    const int64_t Wl = J.Wp[l];
+    if (3 * (Wl - J.Wp[l - 1]) > J.M) return l + 1;
+    int lo = 1, hi = l;
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (3 * (Wl - J.Wp[mid - 1]) <= J.M) hi = mid; else lo = mid + 1;
+    }
+    return lo;
+}
+
 // ---------------------------------------------------------------------------
 // Slab l = 0: A[0][v][p][m] = 0 (T(0,p,t_P,..) = t_P), padding = +inf.
 // ---------------------------------------------------------------------------
@@ -231,7 +246,7 @@ __global__ void __launch_bounds__(kThreads) step_kernel(const Job *__restrict__ 
     }
     if (np <= 0) return;
 
-    const int kmin = kmin_of(J, l);
+    const int kmin = max(kmin_of(J, l), kmin_mem(J, l));
     const int pairs = vcount * np;
     const bool active = tid < pairs;
     const int vv = active ? tid / np : 0;
@@ -422,7 +437,7 @@ __global__ void traceback_kernel(const Job *jobs, int nmp, TraceOut *outs, int32
             continue;
         }
         const double cell = J.table[(size_t)l * slab + (size_t)v * rowlen + (size_t)p * nmp + m];
-        const int km = kmin_of(J, l);
+        const int km = max(kmin_of(J, l), kmin_mem(J, l));
         int code = cell_code_partial(J, nmp, l, p, v, m, cell, km + threadIdx.x, blockDim.x);
         for (int o = 16; o > 0; o >>= 1) code = min(code, __shfl_xor_sync(0xffffffffu, code, o));
         if ((threadIdx.x & 31) == 0) s_code[threadIdx.x >> 5] = code;
@@ -495,7 +510,8 @@ __global__ void argmin_kernel(const Job *job, int nmp, int32_t *arg_out, int L, 
             if (p == 0) {
                 code = 3;
             } else {
-                const int c = cell_code_partial(J, nmp, l, p, v, m, cell, kmin_of(J, l), 1);
+                const int c = cell_code_partial(J, nmp, l, p, v, m, cell,
+                                                max(kmin_of(J, l), kmin_mem(J, l)), 1);
                 code = c == 0x7fffffff ? -2 : c;
             }
         }
