@@ -10,6 +10,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -49,6 +50,7 @@ struct madpipe_ctx {
     int64_t h2d_bytes = 0, d2h_bytes = 0;
     int64_t last_cell_updates = 0, last_effective = 0;
     int per_launch_timing = 0;
+    int use_tma = 1;          // MADPIPE_KERNEL=v1 selects the plain-load step kernel
     std::vector<cudaEvent_t> ev_pool;
 };
 
@@ -213,6 +215,8 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stre
     size_t fr = 0, tot = 0;
     cudaMemGetInfo(&fr, &tot);
     c->mem_budget = mem_budget > 0 ? mem_budget : (int64_t)(0.6 * (double)fr);
+    const char *kern = getenv("MADPIPE_KERNEL");
+    if (kern && strcmp(kern, "v1") == 0) c->use_tma = 0;
     cudaEventCreate(&c->ev_a);
     cudaEventCreate(&c->ev_b);
     *out = c;
@@ -378,6 +382,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         size_t used = 0;
         int maxL = 0;
         size_t max_slab = 0;
+        int smem_tma = 0;
         for (; next < js.size(); next++) {
             const JobSpec &s = js[next];
             if (early_exit && jl_host[s.chain] < s.j) continue;
@@ -396,7 +401,12 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             J.chain = s.chain;
             J.gid = (int32_t)next;
             int n_tiles;
-            tile_geom(c.P, disc->n_delay, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
+            if (ctx->use_tma) {
+                tma_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
+                smem_tma = std::max(smem_tma, tma_smem_bytes(J.vb, J.np, nmp));
+            } else {
+                tile_geom(c.P, disc->n_delay, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
+            }
             J.tile0 = (int32_t)htiles.size();
             for (int t = 0; t < n_tiles; t++) htiles.push_back((int32_t)hjobs.size());
             used += (bytes + 255) & ~(size_t)255;
@@ -432,7 +442,10 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         }
         for (int l = 1; l <= maxL; l++) {
             if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1)], ctx->stream);
-            launch_step(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, ctx->stream);
+            if (ctx->use_tma)
+                launch_step_tma(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, smem_tma, ctx->stream);
+            else
+                launch_step(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, ctx->stream);
             if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1) + 1], ctx->stream);
         }
         ctx->launches += maxL;

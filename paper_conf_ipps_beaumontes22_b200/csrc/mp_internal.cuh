@@ -70,6 +70,10 @@ void launch_jobs_init(Job *jobs, int n_jobs, cudaStream_t s);
 void launch_init_slab0(const Job *jobs, int n_jobs, int nmp, int max_cells, cudaStream_t s);
 void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp,
                  cudaStream_t s);
+void launch_step_tma(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int smem,
+                     cudaStream_t s);
+int tma_smem_bytes(int vb, int np, int nmp);
+void tma_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
 void launch_root(const Job *jobs, int n_jobs, int nmp, int32_t *jl_per_chain, double *root_out,
                  double *tau_out, cudaStream_t s);
 void launch_count(const Job *jobs, int n_jobs, unsigned long long *counts, cudaStream_t s);
