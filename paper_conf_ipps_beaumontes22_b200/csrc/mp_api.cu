@@ -50,7 +50,8 @@ struct madpipe_ctx {
     int64_t h2d_bytes = 0, d2h_bytes = 0;
     int64_t last_cell_updates = 0, last_effective = 0;
     int per_launch_timing = 0;
-    int use_tma = 1;          // MADPIPE_KERNEL=v1 selects the plain-load step kernel
+    int kernel = 2;           // MADPIPE_KERNEL: v1 = plain loads, tma = per-tile TMA, persist (default)
+    int num_sms = 148;
     std::vector<cudaEvent_t> ev_pool;
 };
 
@@ -216,7 +217,9 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stre
     cudaMemGetInfo(&fr, &tot);
     c->mem_budget = mem_budget > 0 ? mem_budget : (int64_t)(0.6 * (double)fr);
     const char *kern = getenv("MADPIPE_KERNEL");
-    if (kern && strcmp(kern, "v1") == 0) c->use_tma = 0;
+    if (kern && strcmp(kern, "v1") == 0) c->kernel = 0;
+    if (kern && strcmp(kern, "tma") == 0) c->kernel = 1;
+    cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device);
     cudaEventCreate(&c->ev_a);
     cudaEventCreate(&c->ev_b);
     *out = c;
@@ -376,19 +379,22 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
     std::vector<int> ids;
     std::vector<unsigned long long> hcounts;
     const size_t budget = (size_t)ctx->mem_budget;
+    // early exit: small first batches that double (time-to-placement); otherwise as
+    // many jobs as the table budget holds
+    size_t cap_jobs = early_exit ? (size_t)8 * (size_t)n_chains : SIZE_MAX;
     while (next < js.size()) {
         // ---- form a batch
         hjobs.clear(); htiles.clear(); ids.clear();
         size_t used = 0;
         int maxL = 0;
         size_t max_slab = 0;
-        int smem_tma = 0;
+        int smem_tma = 0, stage_doubles = 0;
         for (; next < js.size(); next++) {
             const JobSpec &s = js[next];
             if (early_exit && jl_host[s.chain] < s.j) continue;
             const ChainSpec &c = cs[s.chain];
             const size_t bytes = table_doubles(c, disc) * 8;
-            if (!hjobs.empty() && used + bytes > budget) break;
+            if (!hjobs.empty() && (used + bytes > budget || hjobs.size() >= cap_jobs)) break;
             if (hjobs.empty() && bytes > budget && bytes > ctx->tables.n) {
                 // a single job larger than the budget: try anyway (may fail with ENOMEM)
             }
@@ -401,9 +407,10 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             J.chain = s.chain;
             J.gid = (int32_t)next;
             int n_tiles;
-            if (ctx->use_tma) {
+            if (ctx->kernel >= 1) {
                 tma_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
                 smem_tma = std::max(smem_tma, tma_smem_bytes(J.vb, J.np, nmp));
+                stage_doubles = std::max(stage_doubles, J.vb * (J.np + 1) * nmp);
             } else {
                 tile_geom(c.P, disc->n_delay, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
             }
@@ -416,6 +423,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             ids.push_back((int)next);
         }
         if (hjobs.empty()) break;
+        if (cap_jobs != SIZE_MAX) cap_jobs *= 2;
         CUDA_TRY(ctx, ctx->tables.ensure(used));
         for (auto &J : hjobs) J.table = (double *)((char *)ctx->tables.p + (uintptr_t)J.table);
         const int nj = (int)hjobs.size();
@@ -432,6 +440,9 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         launch_init_slab0(djobs, nj, nmp, (int)std::min(max_slab, (size_t)INT32_MAX), ctx->stream);
         ctx->launches += 2;
         const int n_tiles = (int)htiles.size();
+        int persist_grid = 0;
+        if (ctx->kernel == 2)
+            persist_grid = std::min(n_tiles, ctx->num_sms * persist_blocks_per_sm(nmp, stage_doubles));
         const bool per_launch = timed && ctx->per_launch_timing;
         if (per_launch && ctx->ev_pool.size() < (size_t)(2 * maxL)) {
             while (ctx->ev_pool.size() < (size_t)(2 * maxL)) {
@@ -442,7 +453,10 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         }
         for (int l = 1; l <= maxL; l++) {
             if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1)], ctx->stream);
-            if (ctx->use_tma)
+            if (ctx->kernel == 2)
+                launch_step_persist(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, stage_doubles,
+                                    persist_grid, ctx->stream);
+            else if (ctx->kernel == 1)
                 launch_step_tma(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, smem_tma, ctx->stream);
             else
                 launch_step(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, ctx->stream);

@@ -1,0 +1,317 @@
+// mp_step_persist.cu -- the wavefront min-plus step (a3-a5) as a persistent,
+// warp-specialised, TMA-pipelined sm_100a kernel.
+//
+// Same recursion as step_kernel (mp_kernels.cu), P:181-193 in decision form (Q1):
+//   A[l][v][p][m] = clamp_tau( min over live k of
+//        N: A[k-1][v'][p-1][m]            (normal GPU fits)
+//        S: U(k,l) + A[k-1][v'][p][m+d]   (special GPU) ).
+//
+// Structure:
+//   * grid = resident CTAs (a few per SM); CTA c takes tiles c, c+G, c+2G, ...
+//     A tile is vb delay rows x np processor rows of one job (same geometry as
+//     the non-persistent TMA kernel).
+//   * warp 8 is the producer.  For each tile it computes the live transitions
+//     (k, v) of the window with all 32 lanes (a3), writes the base row p = 0
+//     (a4), and for every k with a live row streams the source row segments
+//     A[k-1][v'][p_lo-1 .. p_lo+np-1][*] into an NST-stage shared-memory ring
+//     with cp.async.bulk, completing on the stage's mbarrier.  Per-stage
+//     metadata (the tile's output row, tau, the transition codes, U(k,l))
+//     travels in a small shared-memory array next to the ring.
+//   * warps 0-7 are consumers: each thread owns a (p, m-pair) of one delay row,
+//     so the shift d is warp-uniform.  N is one 16-byte shared load, S one
+//     16-byte (d even) or two 8-byte (d odd) loads + DADD; two min's per level.
+//     At the tile's last stage they clamp to tau and store.
+//   * the ring never drains between tiles, so each SM keeps NST x CTAs row
+//     segments in flight (Little's law for HBM latency).
+// min is exact and order-free, so results equal the oracle's bit for bit.
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "mp_device.cuh"
+#include "mp_internal.cuh"
+
+namespace mp {
+
+namespace {
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred P1;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+        "@!P1 bra WAIT_%=;\n"
+        "}\n" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+
+}  // namespace
+
+constexpr int kPNst = 12;            // ring stages
+constexpr int kPCons = 256;          // consumer threads
+constexpr int kMaxVb = 8;            // delay rows per tile (host geometry caps at this)
+
+// per-stage metadata written by the producer, read by the consumers
+struct StageMeta {
+    double *out;        // output row of delay v0 (row v0+vv at out + vv*rowlen)
+    double tau;
+    double U;           // U(k,l) of this stage's k
+    int32_t tr[kMaxVb]; // transition code per delay row (<0: not live)
+    int32_t rowlen;     // P*NMP
+    int16_t np, vcount, n_m, flags;   // flags: 1 = last stage of the tile, 2 = no data, 4 = terminate
+};
+
+template <int NMP>
+__global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job *__restrict__ jobs,
+                                                                      const int32_t *__restrict__ tile_job,
+                                                                      int n_tiles, int l, int stage_doubles) {
+    constexpr int HP = NMP / 2;
+    extern __shared__ __align__(128) unsigned char dsm[];
+    __shared__ __align__(8) uint64_t full[kPNst];
+    __shared__ __align__(8) uint64_t empty[kPNst];
+    __shared__ StageMeta meta[kPNst];
+    __shared__ Job pJ;              // producer's copy of the current tile's job
+    __shared__ int32_t p_tr[32];
+
+    const int tid = threadIdx.x;
+    const int warp = tid >> 5, lane = tid & 31;
+    if (tid == 0) {
+        for (int s = 0; s < kPNst; s++) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kPCons / 32);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    double *ring = reinterpret_cast<double *>(dsm);
+
+    if (warp == kPCons / 32) {
+        // =================================================== producer warp
+        int gi = 0;
+        for (int tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+            const int jid = tile_job[tile];
+            __syncwarp();
+            if (lane == 0) pJ = jobs[jid];
+            __syncwarp();
+            const Job &J = pJ;
+            const bool alive = l <= J.L;
+            const int t = tile - J.tile0;
+            const int vt = t / J.n_ptiles, pt = t % J.n_ptiles;
+            const int v0 = vt * J.vb;
+            const int vcount = min(J.vb, J.n_v - v0);
+            const int p_lo = 1 + pt * J.np;
+            const int np = max(0, min(J.np, J.P - p_lo));
+            const size_t rowlen = (size_t)J.P * NMP;
+            const size_t slab = (size_t)J.n_v * rowlen;
+            const int seg_doubles = (np + 1) * NMP;
+            const uint32_t seg_bytes = (uint32_t)seg_doubles * 8u;
+            if (!alive) continue;
+            double *out = J.table + (size_t)l * slab;
+            const double Ul = J.Up[l];
+            // base row p = 0 (Q10)
+            if (pt == 0 && lane < vcount) {
+                const int v = v0 + lane;
+                const double U1l = __dsub_rn(Ul, J.Up[0]);
+                int64_t d;
+                (void)transition(J, 1, l, v, U1l, &d);
+                double *o = out + (size_t)v * rowlen;
+#pragma unroll
+                for (int m = 0; m < NMP; m++)
+                    o[m] = (m < J.n_m && U1l <= J.tau && (int64_t)m + d <= (int64_t)(J.n_m - 1)) ? U1l
+                                                                                               : MP_INF;
+            }
+            if (np <= 0) continue;
+            const int kmin = max(kmin_of(J, l), kmin_mem(J, l));
+            const int per = 32 / vcount;            // k per 32-lane pass (vcount <= 8)
+            unsigned long long live_total = 0;
+            for (int kb = kmin; kb <= l; kb += per) {
+                // lane -> (k, vv)
+                const int kk = lane / vcount, v2 = lane - kk * vcount;
+                const int k = kb + kk;
+                int32_t tr = -1;
+                double Ukl = 0.0;
+                if (kk < per && k <= l) {
+                    Ukl = __dsub_rn(Ul, J.Up[k - 1]);
+                    tr = transition(J, k, l, v0 + v2, Ukl, nullptr);
+                }
+                p_tr[lane] = tr;
+                const unsigned live_mask = __ballot_sync(0xffffffffu, tr >= 0);
+                live_total += __popc(live_mask);
+                __syncwarp();
+                if (lane == 0) {
+                    const int nk = min(per, l + 1 - kb);
+                    for (int q = 0; q < nk; q++) {
+                        bool any = false;
+                        uint32_t bytes = 0;
+                        for (int w = 0; w < vcount; w++) {
+                            const bool lv = p_tr[q * vcount + w] >= 0;
+                            any |= lv;
+                            bytes += lv ? seg_bytes : 0u;
+                        }
+                        if (!any) continue;
+                        const int s = gi % kPNst;
+                        if (gi >= kPNst) mbar_wait(&empty[s], (uint32_t)((gi / kPNst - 1) & 1));
+                        StageMeta &M = meta[s];
+                        M.out = out + (size_t)v0 * rowlen + (size_t)p_lo * NMP;
+                        M.tau = J.tau;
+                        M.U = __dsub_rn(Ul, J.Up[kb + q - 1]);
+                        for (int w = 0; w < kMaxVb; w++) M.tr[w] = w < vcount ? p_tr[q * vcount + w] : -1;
+                        M.rowlen = (int32_t)rowlen;
+                        M.np = (int16_t)np; M.vcount = (int16_t)vcount; M.n_m = (int16_t)J.n_m;
+                        M.flags = 0;
+                        mbar_arrive_expect_tx(&full[s], bytes);
+                        const double *src_slab = J.table + (size_t)(kb + q - 1) * slab + (size_t)(p_lo - 1) * NMP;
+                        for (int w = 0; w < vcount; w++) {
+                            const int32_t trw = p_tr[q * vcount + w];
+                            if (trw < 0) continue;
+                            bulk_g2s(ring + (size_t)s * stage_doubles + (size_t)w * seg_doubles,
+                                     src_slab + (size_t)(trw & 0xFFFF) * rowlen, seg_bytes, &full[s]);
+                        }
+                        gi++;
+                    }
+                }
+                __syncwarp();
+                gi = __shfl_sync(0xffffffffu, gi, 0);
+            }
+            if (pt == 0 && lane == 0 && live_total)
+                atomicAdd(J.eff, live_total * (unsigned long long)(J.P - 1) * (unsigned long long)J.n_m);
+            if (lane == 0) {
+                // close the tile with a data-less stage: consumers clamp and store
+                const int s = gi % kPNst;
+                if (gi >= kPNst) mbar_wait(&empty[s], (uint32_t)((gi / kPNst - 1) & 1));
+                StageMeta &M = meta[s];
+                M.out = out + (size_t)v0 * rowlen + (size_t)p_lo * NMP;
+                M.tau = J.tau;
+                M.U = 0.0;
+                for (int w = 0; w < kMaxVb; w++) M.tr[w] = -1;
+                M.rowlen = (int32_t)rowlen;
+                M.np = (int16_t)np; M.vcount = (int16_t)vcount; M.n_m = (int16_t)J.n_m;
+                M.flags = 1 | 2;
+                mbar_arrive(&full[s]);   // no transaction bytes
+                gi++;
+            }
+            gi = __shfl_sync(0xffffffffu, gi, 0);
+        }
+        if (lane == 0) {
+            const int s = gi % kPNst;
+            if (gi >= kPNst) mbar_wait(&empty[s], (uint32_t)((gi / kPNst - 1) & 1));
+            meta[s].flags = 4;
+            mbar_arrive(&full[s]);
+        }
+        return;
+    }
+
+    // ======================================================= consumer warps
+    double best0 = MP_INF, best1 = MP_INF;
+    for (int gi = 0;; gi++) {
+        const int s = gi % kPNst;
+        mbar_wait(&full[s], (uint32_t)((gi / kPNst) & 1));
+        const StageMeta &M = meta[s];
+        const int flags = M.flags;
+        if (flags & 4) break;
+        const int np = M.np, vcount = M.vcount, n_m = M.n_m;
+        const int rowgroup = ((np * HP + 31) / 32) * 32;
+        const int vv = tid / rowgroup;
+        const int q = tid - vv * rowgroup;
+        const int pp_off = q / HP;
+        const int h = q - pp_off * HP;
+        const bool active = vv < vcount && pp_off < np;
+        if (!(flags & 2) && active) {
+            const int32_t tr = M.tr[vv];
+            if (tr >= 0) {
+                const double *seg = ring + (size_t)s * stage_doubles + (size_t)vv * (np + 1) * NMP;
+                if (tr & (1 << 24)) {
+                    const double2 x = *reinterpret_cast<const double2 *>(seg + pp_off * NMP + 2 * h);
+                    best0 = x.x < best0 ? x.x : best0;
+                    best1 = x.y < best1 ? x.y : best1;
+                }
+                const int d = (tr >> 16) & 0xFF;
+                const int m0 = 2 * h + d;
+                if (m0 <= n_m - 1) {
+                    const double U = M.U;
+                    const double *r = seg + (pp_off + 1) * NMP;
+                    double y0, y1;
+                    if ((d & 1) == 0) {
+                        const double2 y = *reinterpret_cast<const double2 *>(r + m0);
+                        y0 = y.x; y1 = y.y;
+                    } else {
+                        y0 = r[m0];
+                        y1 = (m0 + 1 <= n_m - 1) ? r[m0 + 1] : MP_INF;
+                    }
+                    const double c0 = __dadd_rn(U, y0);
+                    best0 = c0 < best0 ? c0 : best0;
+                    if (m0 + 1 <= n_m - 1) {
+                        const double c1 = __dadd_rn(U, y1);
+                        best1 = c1 < best1 ? c1 : best1;
+                    }
+                }
+            }
+        }
+        if (flags & 1) {   // tile complete: clamp (Q12) and store
+            if (active) {
+                double2 r;
+                r.x = (2 * h < n_m && best0 <= M.tau) ? best0 : MP_INF;
+                r.y = (2 * h + 1 < n_m && best1 <= M.tau) ? best1 : MP_INF;
+                *reinterpret_cast<double2 *>(M.out + (size_t)vv * M.rowlen + (size_t)pp_off * NMP + 2 * h) = r;
+            }
+            best0 = MP_INF;
+            best1 = MP_INF;
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[s]);
+    }
+}
+
+int persist_smem_bytes(int stage_doubles) { return kPNst * stage_doubles * 8; }
+
+void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp,
+                         int stage_doubles, int grid, cudaStream_t s) {
+    const int smem = persist_smem_bytes(stage_doubles);
+    switch (nmp) {
+#define MP_CASE(N)                                                                                      \
+    case N:                                                                                             \
+        cudaFuncSetAttribute(step_persist_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
+        step_persist_kernel<N><<<grid, kPCons + 32, smem, s>>>(jobs, tile_job, n_tiles, l, stage_doubles); \
+        break;
+        MP_CASE(2) MP_CASE(4) MP_CASE(8) MP_CASE(16) MP_CASE(32) MP_CASE(64)
+#undef MP_CASE
+    }
+}
+
+int persist_blocks_per_sm(int nmp, int stage_doubles) {
+    const int smem = persist_smem_bytes(stage_doubles);
+    int n = 0;
+    switch (nmp) {
+#define MP_OCC(N)                                                                                       \
+    case N:                                                                                             \
+        cudaFuncSetAttribute(step_persist_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, step_persist_kernel<N>, kPCons + 32, smem);  \
+        break;
+        MP_OCC(2) MP_OCC(4) MP_OCC(8) MP_OCC(16) MP_OCC(32) MP_OCC(64)
+#undef MP_OCC
+    }
+    return n < 1 ? 1 : n;
+}
+
+}  // namespace mp
