@@ -71,6 +71,7 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
 constexpr int kPNst = 12;            // ring stages
 constexpr int kPCons = 256;          // consumer threads
 constexpr int kMaxVb = 8;            // delay rows per tile (host geometry caps at this)
+constexpr int kMaxGroups = 512;      // live k per tile (window <= L <= 512 layers)
 
 // per-stage metadata written by the producer, read by the consumers
 struct StageMeta {
@@ -92,7 +93,8 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
     __shared__ __align__(8) uint64_t empty[kPNst];
     __shared__ StageMeta meta[kPNst];
     __shared__ Job pJ;              // producer's copy of the current tile's job
-    __shared__ int32_t p_tr[32];
+    __shared__ int32_t p_tr[kMaxGroups * kMaxVb];   // live codes of the tile's groups
+    __shared__ int32_t p_grp[kMaxGroups];           // k of each group
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
@@ -108,6 +110,9 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
 
     if (warp == kPCons / 32) {
         // =================================================== producer warp
+        // Phase A (all lanes): live transitions of the tile's window -> p_grp
+        // (compacted k with at least one live delay row) and p_tr (codes).
+        // Phase B (lane-parallel): lane i issues stage gi+i for group i.
         int gi = 0;
         for (int tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
             const int jid = tile_job[tile];
@@ -115,7 +120,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             if (lane == 0) pJ = jobs[jid];
             __syncwarp();
             const Job &J = pJ;
-            const bool alive = l <= J.L;
+            if (l > J.L) continue;
             const int t = tile - J.tile0;
             const int vt = t / J.n_ptiles, pt = t % J.n_ptiles;
             const int v0 = vt * J.vb;
@@ -126,11 +131,11 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             const size_t slab = (size_t)J.n_v * rowlen;
             const int seg_doubles = (np + 1) * NMP;
             const uint32_t seg_bytes = (uint32_t)seg_doubles * 8u;
-            if (!alive) continue;
             double *out = J.table + (size_t)l * slab;
             const double Ul = J.Up[l];
-            // base row p = 0 (Q10)
-            if (pt == 0 && lane < vcount) {
+            const double tau = J.tau;
+            const int n_m = J.n_m;
+            if (pt == 0 && lane < vcount) {       // base row p = 0 (Q10)
                 const int v = v0 + lane;
                 const double U1l = __dsub_rn(Ul, J.Up[0]);
                 int64_t d;
@@ -138,81 +143,98 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                 double *o = out + (size_t)v * rowlen;
 #pragma unroll
                 for (int m = 0; m < NMP; m++)
-                    o[m] = (m < J.n_m && U1l <= J.tau && (int64_t)m + d <= (int64_t)(J.n_m - 1)) ? U1l
-                                                                                               : MP_INF;
+                    o[m] = (m < n_m && U1l <= tau && (int64_t)m + d <= (int64_t)(n_m - 1)) ? U1l : MP_INF;
             }
             if (np <= 0) continue;
+            // ---- phase A
             const int kmin = max(kmin_of(J, l), kmin_mem(J, l));
-            const int per = 32 / vcount;            // k per 32-lane pass (vcount <= 8)
+            const int per = 32 / vcount;                 // k per pass (vcount <= 8)
+            const int kk = lane / vcount, v2 = lane - kk * vcount;
+            const unsigned grp_mask = ((vcount == 32) ? 0xffffffffu : ((1u << vcount) - 1u)) << (kk * vcount);
             unsigned long long live_total = 0;
-            for (int kb = kmin; kb <= l; kb += per) {
-                // lane -> (k, vv)
-                const int kk = lane / vcount, v2 = lane - kk * vcount;
-                const int k = kb + kk;
-                int32_t tr = -1;
-                double Ukl = 0.0;
-                if (kk < per && k <= l) {
-                    Ukl = __dsub_rn(Ul, J.Up[k - 1]);
-                    tr = transition(J, k, l, v0 + v2, Ukl, nullptr);
-                }
-                p_tr[lane] = tr;
-                const unsigned live_mask = __ballot_sync(0xffffffffu, tr >= 0);
-                live_total += __popc(live_mask);
-                __syncwarp();
-                if (lane == 0) {
-                    const int nk = min(per, l + 1 - kb);
-                    for (int q = 0; q < nk; q++) {
-                        bool any = false;
-                        uint32_t bytes = 0;
-                        for (int w = 0; w < vcount; w++) {
-                            const bool lv = p_tr[q * vcount + w] >= 0;
-                            any |= lv;
-                            bytes += lv ? seg_bytes : 0u;
-                        }
-                        if (!any) continue;
-                        const int s = gi % kPNst;
-                        if (gi >= kPNst) mbar_wait(&empty[s], (uint32_t)((gi / kPNst - 1) & 1));
-                        StageMeta &M = meta[s];
-                        M.out = out + (size_t)v0 * rowlen + (size_t)p_lo * NMP;
-                        M.tau = J.tau;
-                        M.U = __dsub_rn(Ul, J.Up[kb + q - 1]);
-                        for (int w = 0; w < kMaxVb; w++) M.tr[w] = w < vcount ? p_tr[q * vcount + w] : -1;
-                        M.rowlen = (int32_t)rowlen;
-                        M.np = (int16_t)np; M.vcount = (int16_t)vcount; M.n_m = (int16_t)J.n_m;
-                        M.flags = 0;
-                        mbar_arrive_expect_tx(&full[s], bytes);
-                        const double *src_slab = J.table + (size_t)(kb + q - 1) * slab + (size_t)(p_lo - 1) * NMP;
-                        for (int w = 0; w < vcount; w++) {
-                            const int32_t trw = p_tr[q * vcount + w];
-                            if (trw < 0) continue;
-                            bulk_g2s(ring + (size_t)s * stage_doubles + (size_t)w * seg_doubles,
-                                     src_slab + (size_t)(trw & 0xFFFF) * rowlen, seg_bytes, &full[s]);
-                        }
-                        gi++;
+            for (int kb = kmin; kb <= l;) {
+                // phase A: collect up to kMaxGroups live groups
+                int ngrp = 0;
+                for (; kb <= l && ngrp + per <= kMaxGroups; kb += per) {
+                    const int k = kb + kk;
+                    int32_t tr = -1;
+                    if (kk < per && k <= l)
+                        tr = transition(J, k, l, v0 + v2, __dsub_rn(Ul, J.Up[k - 1]), nullptr);
+                    const unsigned live = __ballot_sync(0xffffffffu, tr >= 0);
+                    live_total += __popc(live);
+                    const bool valid = kk < per && k <= l;
+                    const bool leader = valid && (v2 == 0) && (live & grp_mask);
+                    const unsigned leaders = __ballot_sync(0xffffffffu, leader);
+                    const int rank = ngrp + __popc(leaders & ((1u << lane) - 1u));
+                    const int myrank = __shfl_sync(0xffffffffu, rank, valid ? kk * vcount : 0);
+                    if (valid && (live & grp_mask)) {
+                        p_tr[myrank * kMaxVb + v2] = tr;
+                        if (v2 == 0) p_grp[myrank] = k;
                     }
+                    ngrp += __popc(leaders);
                 }
+                const bool done = kb > l;
                 __syncwarp();
-                gi = __shfl_sync(0xffffffffu, gi, 0);
+                // phase B: one stage per live group; the tile's last stage carries flag 1
+                // (an empty closing stage if the final chunk has no live group)
+                const int nst = ngrp > 0 ? ngrp : (done ? 1 : 0);
+                for (int g = lane; g < nst; g += 32) {
+                    const int gg = gi + g;
+                    const int s = gg % kPNst;
+                    if (gg >= kPNst) mbar_wait(&empty[s], (uint32_t)((gg / kPNst - 1) & 1));
+                    StageMeta &M = meta[s];
+                    M.out = out + (size_t)v0 * rowlen + (size_t)p_lo * NMP;
+                    M.tau = tau;
+                    M.rowlen = (int32_t)rowlen;
+                    M.np = (int16_t)np; M.vcount = (int16_t)vcount; M.n_m = (int16_t)n_m;
+                    M.flags = (int16_t)((done && g == nst - 1 ? 1 : 0) | (ngrp == 0 ? 2 : 0));
+                    if (ngrp == 0) {
+                        for (int w = 0; w < kMaxVb; w++) M.tr[w] = -1;
+                        M.U = 0.0;
+                        mbar_arrive(&full[s]);
+                        continue;
+                    }
+                    const int k = p_grp[g];
+                    M.U = __dsub_rn(Ul, J.Up[k - 1]);
+                    uint32_t bytes = 0;
+                    for (int w = 0; w < kMaxVb; w++) {
+                        const int32_t trw = w < vcount ? p_tr[g * kMaxVb + w] : -1;
+                        M.tr[w] = trw;
+                        bytes += trw >= 0 ? seg_bytes : 0u;
+                    }
+                    const double *src_slab = J.table + (size_t)(k - 1) * slab + (size_t)(p_lo - 1) * NMP;
+                    for (int w = 0; w < vcount; w++) {
+                        const int32_t trw = p_tr[g * kMaxVb + w];
+                        if (trw < 0) continue;
+                        bulk_g2s(ring + (size_t)s * stage_doubles + (size_t)w * seg_doubles,
+                                 src_slab + (size_t)(trw & 0xFFFF) * rowlen, seg_bytes, &full[s]);
+                    }
+                    mbar_arrive_expect_tx(&full[s], bytes);
+                }
+                gi += nst;
+                __syncwarp();
+                if (done) break;
+            }
+            if (kmin > l) {   // empty window: close the tile
+                if (lane == 0) {
+                    const int s = gi % kPNst;
+                    if (gi >= kPNst) mbar_wait(&empty[s], (uint32_t)((gi / kPNst - 1) & 1));
+                    StageMeta &M = meta[s];
+                    M.out = out + (size_t)v0 * rowlen + (size_t)p_lo * NMP;
+                    M.tau = tau;
+                    M.rowlen = (int32_t)rowlen;
+                    M.np = (int16_t)np; M.vcount = (int16_t)vcount; M.n_m = (int16_t)n_m;
+                    M.flags = 1 | 2;
+                    for (int w = 0; w < kMaxVb; w++) M.tr[w] = -1;
+                    M.U = 0.0;
+                    mbar_arrive(&full[s]);
+                }
+                gi += 1;
             }
             if (pt == 0 && lane == 0 && live_total)
-                atomicAdd(J.eff, live_total * (unsigned long long)(J.P - 1) * (unsigned long long)J.n_m);
-            if (lane == 0) {
-                // close the tile with a data-less stage: consumers clamp and store
-                const int s = gi % kPNst;
-                if (gi >= kPNst) mbar_wait(&empty[s], (uint32_t)((gi / kPNst - 1) & 1));
-                StageMeta &M = meta[s];
-                M.out = out + (size_t)v0 * rowlen + (size_t)p_lo * NMP;
-                M.tau = J.tau;
-                M.U = 0.0;
-                for (int w = 0; w < kMaxVb; w++) M.tr[w] = -1;
-                M.rowlen = (int32_t)rowlen;
-                M.np = (int16_t)np; M.vcount = (int16_t)vcount; M.n_m = (int16_t)J.n_m;
-                M.flags = 1 | 2;
-                mbar_arrive(&full[s]);   // no transaction bytes
-                gi++;
-            }
-            gi = __shfl_sync(0xffffffffu, gi, 0);
+                atomicAdd(J.eff, live_total * (unsigned long long)(J.P - 1) * (unsigned long long)n_m);
         }
+        __syncwarp();
         if (lane == 0) {
             const int s = gi % kPNst;
             if (gi >= kPNst) mbar_wait(&empty[s], (uint32_t)((gi / kPNst - 1) & 1));
@@ -224,6 +246,8 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
 
     // ======================================================= consumer warps
     double best0 = MP_INF, best1 = MP_INF;
+    int cur_np = -1, cur_vc = -1, vv = 0, pp_off = 0, h = 0;
+    bool active = false;
     for (int gi = 0;; gi++) {
         const int s = gi % kPNst;
         mbar_wait(&full[s], (uint32_t)((gi / kPNst) & 1));
@@ -231,12 +255,15 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
         const int flags = M.flags;
         if (flags & 4) break;
         const int np = M.np, vcount = M.vcount, n_m = M.n_m;
-        const int rowgroup = ((np * HP + 31) / 32) * 32;
-        const int vv = tid / rowgroup;
-        const int q = tid - vv * rowgroup;
-        const int pp_off = q / HP;
-        const int h = q - pp_off * HP;
-        const bool active = vv < vcount && pp_off < np;
+        if (np != cur_np || vcount != cur_vc) {
+            const int rowgroup = ((np * HP + 31) / 32) * 32;
+            vv = tid / rowgroup;
+            const int q = tid - vv * rowgroup;
+            pp_off = q / HP;
+            h = q - pp_off * HP;
+            active = vv < vcount && pp_off < np;
+            cur_np = np; cur_vc = vcount;
+        }
         if (!(flags & 2) && active) {
             const int32_t tr = M.tr[vv];
             if (tr >= 0) {
