@@ -178,7 +178,12 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                 // phase B: one stage per live group; the tile's last stage carries flag 1
                 // (an empty closing stage if the final chunk has no live group)
                 const int nst = ngrp > 0 ? ngrp : (done ? 1 : 0);
-                for (int g = lane; g < nst; g += 32) {
+                // rounds of at most kPNst stages: the slots of one round are distinct, so each
+                // lane's parity wait refers to the previous use of its own slot (a lane must
+                // never wait two phases ahead: mbarrier parity would alias)
+                for (int g0 = 0; g0 < nst; g0 += kPNst) {
+                const int g = g0 + lane;
+                if (lane < kPNst && g < nst) {
                     const int gg = gi + g;
                     const int s = gg % kPNst;
                     if (gg >= kPNst) mbar_wait(&empty[s], (uint32_t)((gg / kPNst - 1) & 1));
@@ -192,8 +197,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                         for (int w = 0; w < kMaxVb; w++) M.tr[w] = -1;
                         M.U = 0.0;
                         mbar_arrive(&full[s]);
-                        continue;
-                    }
+                    } else {
                     const int k = p_grp[g];
                     M.U = __dsub_rn(Ul, J.Up[k - 1]);
                     uint32_t bytes = 0;
@@ -210,6 +214,9 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                                  src_slab + (size_t)(trw & 0xFFFF) * rowlen, seg_bytes, &full[s]);
                     }
                     mbar_arrive_expect_tx(&full[s], bytes);
+                    }
+                }
+                __syncwarp();
                 }
                 gi += nst;
                 __syncwarp();
