@@ -43,7 +43,7 @@ struct madpipe_ctx {
     bool own_stream = false;
     int64_t mem_budget = 0;
     std::string err;
-    DevBuf tables, jobs, tiles, chains, chain_data, jl, counts, roots, trace, stages, scratch;
+    DevBuf tables, jobs, tiles, chains, chain_data, jl, counts, roots, trace, stages, scratch, codes;
     cudaEvent_t ev_a = nullptr, ev_b = nullptr;
     double sweep_ms = 0.0, step_ms = 0.0;
     int64_t launches = 0;
@@ -231,7 +231,7 @@ extern "C" void madpipe_ctx_destroy(madpipe_ctx *c) {
     cudaSetDevice(c->device);
     cudaStreamSynchronize(c->stream);
     DevBuf *bufs[] = {&c->tables, &c->jobs, &c->tiles, &c->chains, &c->chain_data, &c->jl,
-                      &c->counts, &c->roots, &c->trace, &c->stages, &c->scratch};
+                      &c->counts, &c->roots, &c->trace, &c->stages, &c->scratch, &c->codes};
     for (DevBuf *b : bufs) b->release();
     for (cudaEvent_t ev : c->ev_pool) cudaEventDestroy(ev);
     if (c->ev_a) cudaEventDestroy(c->ev_a);
@@ -429,8 +429,24 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         const int nj = (int)hjobs.size();
         CUDA_TRY(ctx, ctx->jobs.ensure(sizeof(Job) * nj));
         CUDA_TRY(ctx, ctx->tiles.ensure(sizeof(int32_t) * htiles.size()));
-        CUDA_TRY(ctx, ctx->counts.ensure(sizeof(unsigned long long) * 2 * nj));
-        for (int i = 0; i < nj; i++) hjobs[i].eff = (unsigned long long *)ctx->counts.p + nj + i;
+        CUDA_TRY(ctx, ctx->counts.ensure(sizeof(unsigned long long) * 2 * nj + sizeof(int32_t) * nj));
+        for (int i = 0; i < nj; i++) {
+            hjobs[i].eff = (unsigned long long *)ctx->counts.p + nj + i;
+            hjobs[i].kmin_l = (int32_t *)((unsigned long long *)ctx->counts.p + 2 * nj) + i;
+        }
+        int n_v_max = 0;
+        if (ctx->kernel == 2) {
+            // transition codes of one layer: [job][v][maxL]
+            size_t total = 0;
+            for (auto &J : hjobs) { total += (size_t)J.n_v * (size_t)maxL; n_v_max = std::max(n_v_max, J.n_v); }
+            CUDA_TRY(ctx, ctx->codes.ensure(total * sizeof(int32_t)));
+            size_t off = 0;
+            for (auto &J : hjobs) {
+                J.codes = (int32_t *)ctx->codes.p + off;
+                J.code_cap = maxL;
+                off += (size_t)J.n_v * (size_t)maxL;
+            }
+        }
         Job *djobs = (Job *)ctx->jobs.p;
         CUDA_TRY(ctx, h2d(ctx, djobs, hjobs.data(), sizeof(Job) * nj));
         CUDA_TRY(ctx, h2d(ctx, ctx->tiles.p, htiles.data(), sizeof(int32_t) * htiles.size()));
@@ -453,6 +469,10 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         }
         for (int l = 1; l <= maxL; l++) {
             if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1)], ctx->stream);
+            if (ctx->kernel == 2) {
+                launch_trans(djobs, nj, n_v_max, l, ctx->stream);
+                ctx->launches++;
+            }
             if (ctx->kernel == 2)
                 launch_step_persist(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, stage_doubles,
                                     persist_grid, ctx->stream);

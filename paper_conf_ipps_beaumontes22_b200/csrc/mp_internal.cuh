@@ -42,6 +42,10 @@ struct Job {
     int32_t  gid;       // index of the job in the caller's job list (root/tau export)
     const double *scal; // chain scalars (SC, lb, ub, U(1,L))
     unsigned long long *eff;  // effective (non-skipped) relaxations of this job
+    int32_t *codes;     // [n_v][code_cap] transition codes of layer l, k = kmin_l + kk (persist path)
+    int32_t *kmin_l;    // window start of layer l for this job (written by trans_kernel)
+    int32_t code_cap;   // row capacity of codes (>= longest window of the batch)
+    int32_t pad_;
 };
 
 // Result of a traceback, written by traceback_kernel.
@@ -77,6 +81,7 @@ void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, 
                          int stage_doubles, int grid, cudaStream_t s);
 int persist_blocks_per_sm(int nmp, int stage_doubles);
 void tma_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
+void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, cudaStream_t s);
 void launch_root(const Job *jobs, int n_jobs, int nmp, int32_t *jl_per_chain, double *root_out,
                  double *tau_out, cudaStream_t s);
 void launch_count(const Job *jobs, int n_jobs, unsigned long long *counts, cudaStream_t s);

@@ -252,6 +252,40 @@ void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, i
 }
 
 // ---------------------------------------------------------------------------
+// a3 for the persistent step kernel: every live/dead transition code of layer l,
+// computed by all SMs in parallel (one CTA per job x 8 delay rows) instead of
+// inside the step kernel's producer warp.  codes[v][kk] holds the transition of
+// k = kmin_l + kk; kmin_l = max(kmin_tau, kmin_W).  Also counts
+// the job's effective relaxations.
+// ---------------------------------------------------------------------------
+__global__ void trans_kernel(const Job *jobs, int l) {
+    const Job &J = jobs[blockIdx.y];
+    if (l > J.L) return;
+    const int v0 = blockIdx.x * 8;
+    if (v0 >= J.n_v) return;
+    const int vc = min(8, J.n_v - v0);
+    const int kmin = max(kmin_of(J, l), kmin_mem(J, l));
+    const int wl = l + 1 - kmin;   // may be <= 0
+    if (blockIdx.x == 0 && threadIdx.x == 0) *J.kmin_l = kmin;
+    const double Ul = J.Up[l];
+    unsigned live = 0;
+    for (int e = threadIdx.x; e < vc * max(wl, 0); e += blockDim.x) {
+        const int vv = e / wl, kk = e - vv * wl;
+        const int k = kmin + kk;
+        const int32_t tr = transition(J, k, l, v0 + vv, __dsub_rn(Ul, J.Up[k - 1]), nullptr);
+        J.codes[(size_t)(v0 + vv) * J.code_cap + kk] = tr;
+        live += tr >= 0;
+    }
+    for (int o = 16; o > 0; o >>= 1) live += __shfl_xor_sync(0xffffffffu, live, o);
+    if ((threadIdx.x & 31) == 0 && live && J.P > 1)
+        atomicAdd(J.eff, (unsigned long long)live * (unsigned long long)(J.P - 1) * (unsigned long long)J.n_m);
+}
+
+void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, cudaStream_t s) {
+    trans_kernel<<<dim3((n_v_max + 7) / 8, n_jobs), 256, 0, s>>>(jobs, l);
+}
+
+// ---------------------------------------------------------------------------
 // a6: root test.  feasible_j = A_j[L][P-1][0][0] <= tau_j (O7); the smallest
 // feasible j of each chain is kept with atomicMin.
 // ---------------------------------------------------------------------------

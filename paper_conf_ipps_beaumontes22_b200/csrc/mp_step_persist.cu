@@ -146,23 +146,21 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                     o[m] = (m < n_m && U1l <= tau && (int64_t)m + d <= (int64_t)(n_m - 1)) ? U1l : MP_INF;
             }
             if (np <= 0) continue;
-            // ---- phase A
-            const int kmin = max(kmin_of(J, l), kmin_mem(J, l));
+            // ---- phase A: read the precomputed codes of the window (trans_kernel)
+            const int kmin = *J.kmin_l;
+            const int wl = l + 1 - kmin;
             const int per = 32 / vcount;                 // k per pass (vcount <= 8)
             const int kk = lane / vcount, v2 = lane - kk * vcount;
-            const unsigned grp_mask = ((vcount == 32) ? 0xffffffffu : ((1u << vcount) - 1u)) << (kk * vcount);
-            unsigned long long live_total = 0;
+            const unsigned grp_mask = ((1u << vcount) - 1u) << (kk * vcount);
+            const int32_t *codes = J.codes + (size_t)(v0 + v2) * J.code_cap;
             for (int kb = kmin; kb <= l;) {
-                // phase A: collect up to kMaxGroups live groups
+                // collect up to kMaxGroups live groups
                 int ngrp = 0;
                 for (; kb <= l && ngrp + per <= kMaxGroups; kb += per) {
                     const int k = kb + kk;
-                    int32_t tr = -1;
-                    if (kk < per && k <= l)
-                        tr = transition(J, k, l, v0 + v2, __dsub_rn(Ul, J.Up[k - 1]), nullptr);
-                    const unsigned live = __ballot_sync(0xffffffffu, tr >= 0);
-                    live_total += __popc(live);
                     const bool valid = kk < per && k <= l;
+                    const int32_t tr = valid ? codes[k - kmin] : -1;
+                    const unsigned live = __ballot_sync(0xffffffffu, tr >= 0);
                     const bool leader = valid && (v2 == 0) && (live & grp_mask);
                     const unsigned leaders = __ballot_sync(0xffffffffu, leader);
                     const int rank = ngrp + __popc(leaders & ((1u << lane) - 1u));
@@ -222,6 +220,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                 __syncwarp();
                 if (done) break;
             }
+            (void)wl;
             if (kmin > l) {   // empty window: close the tile
                 if (lane == 0) {
                     const int s = gi % kPNst;
@@ -238,8 +237,6 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                 }
                 gi += 1;
             }
-            if (pt == 0 && lane == 0 && live_total)
-                atomicAdd(J.eff, live_total * (unsigned long long)(J.P - 1) * (unsigned long long)n_m);
         }
         __syncwarp();
         if (lane == 0) {
