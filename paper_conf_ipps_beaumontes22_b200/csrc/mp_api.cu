@@ -410,7 +410,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             if (ctx->kernel >= 1) {
                 tma_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
                 smem_tma = std::max(smem_tma, tma_smem_bytes(J.vb, J.np, nmp));
-                stage_doubles = std::max(stage_doubles, J.vb * (J.np + 1) * nmp);
+                stage_doubles = std::max(stage_doubles, persist_group_rows() * J.vb * (J.np + 1) * nmp);
             } else {
                 tile_geom(c.P, disc->n_delay, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
             }

@@ -68,19 +68,21 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
 
 }  // namespace
 
-constexpr int kPNst = 12;            // ring stages
+constexpr int kPNst = 8;             // ring stages
+constexpr int kG = 4;                // source k-rows (x delay rows) per stage
 constexpr int kPCons = 256;          // consumer threads
 constexpr int kMaxVb = 8;            // delay rows per tile (host geometry caps at this)
 constexpr int kMaxGroups = 512;      // live k per tile (window <= L <= 512 layers)
 
 // per-stage metadata written by the producer, read by the consumers
 struct StageMeta {
-    double *out;        // output row of delay v0 (row v0+vv at out + vv*rowlen)
+    double *out;              // output row of delay v0 (row v0+vv at out + vv*rowlen)
     double tau;
-    double U;           // U(k,l) of this stage's k
-    int32_t tr[kMaxVb]; // transition code per delay row (<0: not live)
-    int32_t rowlen;     // P*NMP
+    double U[kG];             // U(k,l) of each k of the stage
+    int32_t tr[kG][kMaxVb];   // transition code per (k, delay row) (<0: not live)
+    int32_t rowlen;           // P*NMP
     int16_t np, vcount, n_m, flags;   // flags: 1 = last stage of the tile, 2 = no data, 4 = terminate
+    int16_t ng, pad_[3];      // k-rows in this stage
 };
 
 template <int NMP>
@@ -173,51 +175,52 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                 }
                 const bool done = kb > l;
                 __syncwarp();
-                // phase B: one stage per live group; the tile's last stage carries flag 1
-                // (an empty closing stage if the final chunk has no live group)
-                const int nst = ngrp > 0 ? ngrp : (done ? 1 : 0);
-                // rounds of at most kPNst stages: the slots of one round are distinct, so each
-                // lane's parity wait refers to the previous use of its own slot (a lane must
-                // never wait two phases ahead: mbarrier parity would alias)
+                // phase B: stages of up to kG live groups; the tile's last stage carries
+                // flag 1 (an empty closing stage if the final chunk has no live group).
+                // Rounds of at most kPNst stages: the slots of one round are distinct, so
+                // each lane's parity wait refers to the previous use of its own slot (a
+                // lane must never wait two phases ahead: mbarrier parity would alias).
+                const int nst = ngrp > 0 ? (ngrp + kG - 1) / kG : (done ? 1 : 0);
                 for (int g0 = 0; g0 < nst; g0 += kPNst) {
-                const int g = g0 + lane;
-                if (lane < kPNst && g < nst) {
-                    const int gg = gi + g;
-                    const int s = gg % kPNst;
-                    if (gg >= kPNst) mbar_wait(&empty[s], (uint32_t)((gg / kPNst - 1) & 1));
-                    StageMeta &M = meta[s];
-                    M.out = out + (size_t)v0 * rowlen + (size_t)p_lo * NMP;
-                    M.tau = tau;
-                    M.rowlen = (int32_t)rowlen;
-                    M.np = (int16_t)np; M.vcount = (int16_t)vcount; M.n_m = (int16_t)n_m;
-                    M.flags = (int16_t)((done && g == nst - 1 ? 1 : 0) | (ngrp == 0 ? 2 : 0));
-                    if (ngrp == 0) {
-                        for (int w = 0; w < kMaxVb; w++) M.tr[w] = -1;
-                        M.U = 0.0;
-                        mbar_arrive(&full[s]);
-                    } else {
-                    const int k = p_grp[g];
-                    M.U = __dsub_rn(Ul, J.Up[k - 1]);
-                    uint32_t bytes = 0;
-                    for (int w = 0; w < kMaxVb; w++) {
-                        const int32_t trw = w < vcount ? p_tr[g * kMaxVb + w] : -1;
-                        M.tr[w] = trw;
-                        bytes += trw >= 0 ? seg_bytes : 0u;
+                    const int g = g0 + lane;
+                    if (lane < kPNst && g < nst) {
+                        const int gg = gi + g;
+                        const int s = gg % kPNst;
+                        if (gg >= kPNst) mbar_wait(&empty[s], (uint32_t)((gg / kPNst - 1) & 1));
+                        StageMeta &M = meta[s];
+                        M.out = out + (size_t)v0 * rowlen + (size_t)p_lo * NMP;
+                        M.tau = tau;
+                        M.rowlen = (int32_t)rowlen;
+                        M.np = (int16_t)np; M.vcount = (int16_t)vcount; M.n_m = (int16_t)n_m;
+                        M.flags = (int16_t)((done && g == nst - 1 ? 1 : 0) | (ngrp == 0 ? 2 : 0));
+                        if (ngrp == 0) {
+                            M.ng = 0;
+                            mbar_arrive(&full[s]);
+                        } else {
+                            const int q0 = g * kG;
+                            const int ng = min(kG, ngrp - q0);
+                            M.ng = (int16_t)ng;
+                            uint32_t bytes = 0;
+                            for (int q = 0; q < ng; q++) {
+                                const int k = p_grp[q0 + q];
+                                M.U[q] = __dsub_rn(Ul, J.Up[k - 1]);
+                                const double *src_slab =
+                                    J.table + (size_t)(k - 1) * slab + (size_t)(p_lo - 1) * NMP;
+                                for (int w = 0; w < kMaxVb; w++) {
+                                    const int32_t trw = w < vcount ? p_tr[(q0 + q) * kMaxVb + w] : -1;
+                                    M.tr[q][w] = trw;
+                                    if (trw < 0) continue;
+                                    bytes += seg_bytes;
+                                    bulk_g2s(ring + (size_t)s * stage_doubles + (size_t)(q * vcount + w) * seg_doubles,
+                                             src_slab + (size_t)(trw & 0xFFFF) * rowlen, seg_bytes, &full[s]);
+                                }
+                            }
+                            mbar_arrive_expect_tx(&full[s], bytes);
+                        }
                     }
-                    const double *src_slab = J.table + (size_t)(k - 1) * slab + (size_t)(p_lo - 1) * NMP;
-                    for (int w = 0; w < vcount; w++) {
-                        const int32_t trw = p_tr[g * kMaxVb + w];
-                        if (trw < 0) continue;
-                        bulk_g2s(ring + (size_t)s * stage_doubles + (size_t)w * seg_doubles,
-                                 src_slab + (size_t)(trw & 0xFFFF) * rowlen, seg_bytes, &full[s]);
-                    }
-                    mbar_arrive_expect_tx(&full[s], bytes);
-                    }
-                }
-                __syncwarp();
+                    __syncwarp();
                 }
                 gi += nst;
-                __syncwarp();
                 if (done) break;
             }
             (void)wl;
@@ -231,8 +234,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                     M.rowlen = (int32_t)rowlen;
                     M.np = (int16_t)np; M.vcount = (int16_t)vcount; M.n_m = (int16_t)n_m;
                     M.flags = 1 | 2;
-                    for (int w = 0; w < kMaxVb; w++) M.tr[w] = -1;
-                    M.U = 0.0;
+                    M.ng = 0;
                     mbar_arrive(&full[s]);
                 }
                 gi += 1;
@@ -269,9 +271,11 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             cur_np = np; cur_vc = vcount;
         }
         if (!(flags & 2) && active) {
-            const int32_t tr = M.tr[vv];
-            if (tr >= 0) {
-                const double *seg = ring + (size_t)s * stage_doubles + (size_t)vv * (np + 1) * NMP;
+            const int ng = M.ng;
+            for (int q = 0; q < ng; q++) {
+                const int32_t tr = M.tr[q][vv];
+                if (tr < 0) continue;
+                const double *seg = ring + (size_t)s * stage_doubles + (size_t)(q * vcount + vv) * (np + 1) * NMP;
                 if (tr & (1 << 24)) {
                     const double2 x = *reinterpret_cast<const double2 *>(seg + pp_off * NMP + 2 * h);
                     best0 = x.x < best0 ? x.x : best0;
@@ -280,7 +284,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                 const int d = (tr >> 16) & 0xFF;
                 const int m0 = 2 * h + d;
                 if (m0 <= n_m - 1) {
-                    const double U = M.U;
+                    const double U = M.U[q];
                     const double *r = seg + (pp_off + 1) * NMP;
                     double y0, y1;
                     if ((d & 1) == 0) {
@@ -313,6 +317,8 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
         if (lane == 0) mbar_arrive(&empty[s]);
     }
 }
+
+int persist_group_rows() { return kG; }
 
 int persist_smem_bytes(int stage_doubles) { return kPNst * stage_doubles * 8; }
 
