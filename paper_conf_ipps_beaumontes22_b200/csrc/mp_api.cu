@@ -407,10 +407,12 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             J.chain = s.chain;
             J.gid = (int32_t)next;
             int n_tiles;
-            if (ctx->kernel >= 1) {
+            if (ctx->kernel == 2) {
+                persist_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
+                stage_doubles = std::max(stage_doubles, J.vb * (J.np + 1) * nmp);
+            } else if (ctx->kernel == 1) {
                 tma_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
                 smem_tma = std::max(smem_tma, tma_smem_bytes(J.vb, J.np, nmp));
-                stage_doubles = std::max(stage_doubles, persist_group_rows() * J.vb * (J.np + 1) * nmp);
             } else {
                 tile_geom(c.P, disc->n_delay, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
             }
@@ -456,9 +458,12 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         launch_init_slab0(djobs, nj, nmp, (int)std::min(max_slab, (size_t)INT32_MAX), ctx->stream);
         ctx->launches += 2;
         const int n_tiles = (int)htiles.size();
-        int persist_grid = 0;
-        if (ctx->kernel == 2)
-            persist_grid = std::min(n_tiles, ctx->num_sms * persist_blocks_per_sm(nmp, stage_doubles));
+        int persist_grid = 0, nst = 0;
+        if (ctx->kernel == 2) {
+            nst = persist_nst(stage_doubles);
+            if (nst < 2) return fail(ctx, MADPIPE_EINVAL, "row segment too large for the step kernel ring");
+            persist_grid = std::min(n_tiles, ctx->num_sms * persist_blocks_per_sm(nmp, stage_doubles, nst));
+        }
         const bool per_launch = timed && ctx->per_launch_timing;
         if (per_launch && ctx->ev_pool.size() < (size_t)(2 * maxL)) {
             while (ctx->ev_pool.size() < (size_t)(2 * maxL)) {
@@ -474,7 +479,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 ctx->launches++;
             }
             if (ctx->kernel == 2)
-                launch_step_persist(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, stage_doubles,
+                launch_step_persist(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, stage_doubles, nst,
                                     persist_grid, ctx->stream);
             else if (ctx->kernel == 1)
                 launch_step_tma(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, smem_tma, ctx->stream);
