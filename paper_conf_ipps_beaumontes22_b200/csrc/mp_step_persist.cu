@@ -70,7 +70,7 @@ __device__ __forceinline__ double dmin(double a, double b) { return b < a ? b : 
 constexpr int kNstMax = 12;          // ring stages (runtime nst <= kNstMax)
 constexpr int kPCons = 256;          // consumer threads (8 warps); + 1 producer warp
 constexpr int kMaxVb = 8;            // delay rows per tile
-constexpr int kMaxGroups = 512;      // live k collected per producer round
+constexpr int kMaxGroups = 128;      // live k collected per producer round
 
 // per-stage metadata written by the producer, read by the consumers
 struct StageMeta {
@@ -374,7 +374,7 @@ void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int 
 
 // ring depth that fits in ~100 KB of dynamic shared memory (2 CTAs per SM)
 int persist_nst(int stage_doubles) {
-    int n = (100 * 1024) / (stage_doubles * 8);
+    int n = (96 * 1024) / (stage_doubles * 8);
     if (n > kNstMax) n = kNstMax;
     return n;   // the caller falls back to another step kernel if n < 2
 }
