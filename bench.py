@@ -202,8 +202,8 @@ def main():
         else:
             res, cu = solve_distributed(chain, *a, early_exit=early_exit, ctx=ctx, device=dev)
         t = ctx.last_timing()
-        eff = ctx.last_counts()["effective_updates"]
-        return res, cu, eff, t["launches"], t["step_ms"]
+        cnt = ctx.last_counts()
+        return res, cu, (cnt["effective_updates"], cnt["useful_updates"]), t["launches"], t["step_ms"]
 
     def timed(chain, k, early_exit=False):
         dev_ms, wall, cus, effs, launches, kern_ms, io = [], [], [], [], 0, 0.0, (0, 0)
@@ -250,7 +250,8 @@ def main():
     K = args.steps
     tot_ms = reduce(sum(main_run["dev_ms"]), MAX)
     cu_step = reduce(main_run["cu"][-1], SUM)
-    eff_step = reduce(main_run["eff"][-1], SUM)
+    eff_step = reduce(main_run["eff"][-1][0], SUM)
+    useful_step = reduce(main_run["eff"][-1][1], SUM)
     value = cu_step * K / (tot_ms / 1e3)
     kern_ms = reduce(main_run["kern_ms"], MAX)
     launches = int(reduce(main_run["launches"], SUM))
@@ -272,9 +273,11 @@ def main():
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) \
         if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
     hbm_peak = peaks.get("hbm_gbs", 6650.0)
-    # algorithmic bytes: one fp64 source value per EFFECTIVE relaxation (a live transition
-    # reads the table; skipped ones -- delay overflow, C > tau -- read nothing)
-    achieved = eff_step * K * BYTES_PER_UPDATE / (kern_ms / 1e3) / 1e9 if kern_ms > 0 else None
+    # algorithmic bytes: one fp64 source value per relaxation that must read the table:
+    # a live transition (not skipped by delay overflow / C > tau / no fit) whose source row
+    # holds a finite value; all-+inf rows and dead transitions read nothing
+    units = useful_step if useful_step > 0 else eff_step
+    achieved = units * K * BYTES_PER_UPDATE / (kern_ms / 1e3) / 1e9 if kern_ms > 0 else None
     traffic = None
     prof = os.path.join(ROOT, "profiles", "step_kernel_traffic.json")
     if os.path.exists(prof):
@@ -296,12 +299,15 @@ def main():
         "cell_updates_per_step": cu_step,
         "effective_updates_per_step": eff_step,
         "effective_updates_per_s": eff_step * K / (tot_ms / 1e3),
+        "useful_updates_per_step": useful_step,
         "result": {"cand_index": res["cand_index"], "period": res["period"],
                    "special_load": res["special_load"], "n_stages": len(res["stages"])},
         "roofline": {"bound": "hbm", "kernel": "step_kernel", "achieved": achieved, "peak": hbm_peak,
                      "unit": "GB/s", "frac": (achieved / hbm_peak) if achieved else None,
                      "traffic": traffic, "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)",
-                     "bytes_per_update": BYTES_PER_UPDATE, "units": "effective relaxations",
+                     "bytes_per_update": BYTES_PER_UPDATE,
+                     "units": "useful relaxations (live transition, finite source row)"
+                     if useful_step > 0 else "effective relaxations",
                      "kernel_share": kern_ms / tot_ms if tot_ms else None},
         "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(), "cpu_baseline": cpu,
     }

@@ -177,12 +177,37 @@ int madpipe_set_timing(madpipe_ctx *ctx, int per_launch);
 /* Bytes the last call copied host->device and device->host (inputs, job
  * descriptors, results); for the bench's end-to-end record. */
 int madpipe_last_io(const madpipe_ctx *ctx, int64_t *h2d_bytes, int64_t *d2h_bytes);
-/* Relaxation counts of the last sweep: cell_updates as in madpipe_alloc (every
- * (k, l, v, p, m) of the windows) and effective_updates, the
- * relaxations whose transition is live (not skipped by a delay overflow, a
- * communication longer than the period, or neither N nor S fitting) -- the
- * ones that read the DP table. */
-int madpipe_last_counts(const madpipe_ctx *ctx, int64_t *cell_updates, int64_t *effective_updates);
+/* Relaxation counts of the last sweep: cell_updates as in
+ * madpipe_alloc (every (k, l, v, p, m) of the tau-windows); effective_updates,
+ * the relaxations whose transition is live (not skipped by a delay overflow, a
+ * communication longer than the period, or neither N nor S fitting); and
+ * useful_updates, the live ones whose source row holds a finite value -- the
+ * ones the default step kernel reads (0 for the other step kernels). */
+int madpipe_last_counts(const madpipe_ctx *ctx, int64_t *cell_updates, int64_t *effective_updates,
+                        int64_t *useful_updates);
+
+/* ---- NEXT row f2: the 1F1B* pattern of a contiguous allocation (host only) --
+ * For stages s_1..s_N (one per GPU, tiling layers 1..L in order; e.g. a
+ * madpipe_alloc whose special GPU holds at most one stage) and a period T:
+ * the 2N-1 item chain of stages and communications, its 1F1B* groups
+ * and the periodic pattern: for every item its forward and
+ * backward start time in [0, T), index shift h (in period k the operation
+ * processes batch k-h) and duration.  Item i of group g keeps g activations
+ * alive.  ops[] is caller-allocated with capacity 2N-1.
+ * Returns MADPIPE_INFEASIBLE if an item's load exceeds T, MADPIPE_EINVAL for
+ * stages that do not tile the chain. */
+typedef struct {
+    int32_t kind;       /* 0 = stage (GPU), 1 = communication (link)                 */
+    int32_t stage;      /* stage index (for a communication: the stage it feeds)      */
+    int32_t group;      /* 1F1B* group, 1 = the group holding the last stage          */
+    int32_t f_shift;    /* index shift of the forward operation                       */
+    int32_t b_shift;    /* index shift of the backward operation                      */
+    int32_t pad_;
+    double  f_start, f_len, b_start, b_len;   /* seconds; starts in [0, T)             */
+} madpipe_op;
+int madpipe_schedule(const madpipe_chain *chain, double beta, double period, int32_t n_stages,
+                     const int32_t *stage_first, const int32_t *stage_last, madpipe_op *ops,
+                     int32_t *n_ops);
 
 #ifdef __cplusplus
 }

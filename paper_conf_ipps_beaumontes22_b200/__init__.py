@@ -15,7 +15,7 @@ import numpy as np
 from . import _native as N
 from ._native import VRANGE_PAPER, VRANGE_SAFE, MadpipeError  # noqa: F401
 
-__all__ = ["Context", "validate", "shard", "cell_updates", "VRANGE_PAPER", "VRANGE_SAFE",
+__all__ = ["Context", "validate", "shard", "cell_updates", "schedule", "VRANGE_PAPER", "VRANGE_SAFE",
            "MadpipeError"]
 
 
@@ -38,6 +38,27 @@ def cell_updates(chain, P, n_mem, n_delay, tau) -> int:
     hc = N.HostChain(chain)
     d = N.make_disc(n_mem, n_delay, 1)
     return int(N.lib().madpipe_cell_updates(ctypes.byref(hc.c), int(P), ctypes.byref(d), float(tau)))
+
+
+def schedule(chain, beta, period, stages):
+    """madpipe_schedule (host only): the 1F1B* pattern of a contiguous allocation
+    (P:101-113).  ``stages`` = [(first, last, ...), ...] in chain order.
+    Returns a list of dicts (kind 'stage'/'comm', stage, group, F=(start, shift),
+    B=(start, shift), f_len, b_len), or None if an item exceeds the period."""
+    hc = N.HostChain(chain)
+    first = np.ascontiguousarray([s[0] for s in stages], np.int32)
+    last = np.ascontiguousarray([s[1] for s in stages], np.int32)
+    ops = (N.Op * (2 * len(stages) - 1))()
+    n = ctypes.c_int32()
+    rc = N.lib().madpipe_schedule(ctypes.byref(hc.c), float(beta), float(period), len(stages),
+                                  first.ctypes.data_as(N._i32p), last.ctypes.data_as(N._i32p), ops,
+                                  ctypes.byref(n))
+    if rc == N.INFEASIBLE:
+        return None
+    N.check(rc)
+    return [dict(kind="comm" if o.kind else "stage", stage=o.stage, group=o.group,
+                 F=(o.f_start, o.f_shift), B=(o.b_start, o.b_shift), f_len=o.f_len, b_len=o.b_len)
+            for o in ops[:n.value]]
 
 
 class _DevChain:
@@ -183,9 +204,9 @@ class Context:
         return dict(h2d_bytes=a.value, d2h_bytes=b.value)
 
     def last_counts(self):
-        a = ctypes.c_int64(); b = ctypes.c_int64()
-        N.check(self._lib.madpipe_last_counts(self.h, ctypes.byref(a), ctypes.byref(b)))
-        return dict(cell_updates=a.value, effective_updates=b.value)
+        a = ctypes.c_int64(); b = ctypes.c_int64(); c = ctypes.c_int64()
+        N.check(self._lib.madpipe_last_counts(self.h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)))
+        return dict(cell_updates=a.value, effective_updates=b.value, useful_updates=c.value)
 
     def last_timing(self):
         s = ctypes.c_double(); k = ctypes.c_double(); n = ctypes.c_int64()

@@ -30,6 +30,13 @@ class Disc(ctypes.Structure):
                 ("early_exit", ctypes.c_int32)]
 
 
+class Op(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("stage", ctypes.c_int32), ("group", ctypes.c_int32),
+                ("f_shift", ctypes.c_int32), ("b_shift", ctypes.c_int32), ("pad_", ctypes.c_int32),
+                ("f_start", ctypes.c_double), ("f_len", ctypes.c_double), ("b_start", ctypes.c_double),
+                ("b_len", ctypes.c_double)]
+
+
 class Alloc(ctypes.Structure):
     _fields_ = [("period", ctypes.c_double), ("load_period", ctypes.c_double),
                 ("special_load", ctypes.c_double), ("cand_index", ctypes.c_int32),
@@ -74,7 +81,9 @@ def lib():
         "madpipe_last_timing": (ctypes.c_int, [vp, _dp, _dp, _i64p]),
         "madpipe_set_timing": (ctypes.c_int, [vp, ctypes.c_int]),
         "madpipe_last_io": (ctypes.c_int, [vp, _i64p, _i64p]),
-        "madpipe_last_counts": (ctypes.c_int, [vp, _i64p, _i64p]),
+        "madpipe_last_counts": (ctypes.c_int, [vp, _i64p, _i64p, _i64p]),
+        "madpipe_schedule": (ctypes.c_int, [cp, ctypes.c_double, ctypes.c_double, ctypes.c_int32, _i32p, _i32p,
+                                            ctypes.POINTER(Op), _i32p]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -88,7 +97,7 @@ EXPORTED = ["madpipe_ctx_create", "madpipe_ctx_destroy", "madpipe_last_error", "
             "madpipe_shard", "madpipe_cell_updates", "madpipe_solve", "madpipe_solve_dev",
             "madpipe_sweep", "madpipe_resolve", "madpipe_solve_batch", "madpipe_candidates",
             "madpipe_dp_table", "madpipe_last_timing", "madpipe_set_timing", "madpipe_last_io",
-            "madpipe_last_counts"]
+            "madpipe_last_counts", "madpipe_schedule"]
 
 
 class MadpipeError(RuntimeError):

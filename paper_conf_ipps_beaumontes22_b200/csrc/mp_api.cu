@@ -43,12 +43,12 @@ struct madpipe_ctx {
     bool own_stream = false;
     int64_t mem_budget = 0;
     std::string err;
-    DevBuf tables, jobs, tiles, chains, chain_data, jl, counts, roots, trace, stages, scratch, codes;
+    DevBuf tables, jobs, tiles, chains, chain_data, jl, counts, roots, trace, stages, scratch, codes, flags;
     cudaEvent_t ev_a = nullptr, ev_b = nullptr;
     double sweep_ms = 0.0, step_ms = 0.0;
     int64_t launches = 0;
     int64_t h2d_bytes = 0, d2h_bytes = 0;
-    int64_t last_cell_updates = 0, last_effective = 0;
+    int64_t last_cell_updates = 0, last_effective = 0, last_useful = 0;
     int per_launch_timing = 0;
     int kernel = 2;           // MADPIPE_KERNEL: v1 = plain loads, tma = per-tile TMA, persist (default)
     int num_sms = 148;
@@ -231,7 +231,7 @@ extern "C" void madpipe_ctx_destroy(madpipe_ctx *c) {
     cudaSetDevice(c->device);
     cudaStreamSynchronize(c->stream);
     DevBuf *bufs[] = {&c->tables, &c->jobs, &c->tiles, &c->chains, &c->chain_data, &c->jl,
-                      &c->counts, &c->roots, &c->trace, &c->stages, &c->scratch, &c->codes};
+                      &c->counts, &c->roots, &c->trace, &c->stages, &c->scratch, &c->codes, &c->flags};
     for (DevBuf *b : bufs) b->release();
     for (cudaEvent_t ev : c->ev_pool) cudaEventDestroy(ev);
     if (c->ev_a) cudaEventDestroy(c->ev_a);
@@ -250,10 +250,11 @@ extern "C" int madpipe_last_timing(const madpipe_ctx *c, double *sweep_ms, doubl
 }
 
 extern "C" int madpipe_last_counts(const madpipe_ctx *c, int64_t *cell_updates,
-                                   int64_t *effective_updates) {
+                                   int64_t *effective_updates, int64_t *useful_updates) {
     if (!c) return MADPIPE_EINVAL;
     if (cell_updates) *cell_updates = c->last_cell_updates;
     if (effective_updates) *effective_updates = c->last_effective;
+    if (useful_updates) *useful_updates = c->last_useful;
     return MADPIPE_OK;
 }
 
@@ -372,7 +373,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
     size_t next = 0;
     if (timed) {
         ctx->sweep_ms = 0.0; ctx->step_ms = 0.0;
-        ctx->last_cell_updates = 0; ctx->last_effective = 0;
+        ctx->last_cell_updates = 0; ctx->last_effective = 0; ctx->last_useful = 0;
     }
     std::vector<Job> hjobs;
     std::vector<int32_t> htiles;
@@ -431,10 +432,11 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         const int nj = (int)hjobs.size();
         CUDA_TRY(ctx, ctx->jobs.ensure(sizeof(Job) * nj));
         CUDA_TRY(ctx, ctx->tiles.ensure(sizeof(int32_t) * htiles.size()));
-        CUDA_TRY(ctx, ctx->counts.ensure(sizeof(unsigned long long) * 2 * nj + sizeof(int32_t) * nj));
+        CUDA_TRY(ctx, ctx->counts.ensure(sizeof(unsigned long long) * 3 * nj + sizeof(int32_t) * nj));
         for (int i = 0; i < nj; i++) {
             hjobs[i].eff = (unsigned long long *)ctx->counts.p + nj + i;
-            hjobs[i].kmin_l = (int32_t *)((unsigned long long *)ctx->counts.p + 2 * nj) + i;
+            hjobs[i].useful = (unsigned long long *)ctx->counts.p + 2 * nj + i;
+            hjobs[i].kmin_l = (int32_t *)((unsigned long long *)ctx->counts.p + 3 * nj) + i;
         }
         int n_v_max = 0;
         if (ctx->kernel == 2) {
@@ -442,17 +444,24 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             size_t total = 0;
             for (auto &J : hjobs) { total += (size_t)J.n_v * (size_t)maxL; n_v_max = std::max(n_v_max, J.n_v); }
             CUDA_TRY(ctx, ctx->codes.ensure(total * sizeof(int32_t)));
-            size_t off = 0;
+            size_t off = 0, ftotal = 0;
             for (auto &J : hjobs) {
                 J.codes = (int32_t *)ctx->codes.p + off;
                 J.code_cap = maxL;
                 off += (size_t)J.n_v * (size_t)maxL;
+                ftotal += (size_t)(J.L + 1) * (size_t)J.n_v;
+            }
+            CUDA_TRY(ctx, ctx->flags.ensure(ftotal * sizeof(uint32_t)));
+            size_t foff = 0;
+            for (auto &J : hjobs) {
+                J.rowflag = (uint32_t *)ctx->flags.p + foff;
+                foff += (size_t)(J.L + 1) * (size_t)J.n_v;
             }
         }
         Job *djobs = (Job *)ctx->jobs.p;
         CUDA_TRY(ctx, h2d(ctx, djobs, hjobs.data(), sizeof(Job) * nj));
         CUDA_TRY(ctx, h2d(ctx, ctx->tiles.p, htiles.data(), sizeof(int32_t) * htiles.size()));
-        CUDA_TRY(ctx, cudaMemsetAsync(ctx->counts.p, 0, sizeof(unsigned long long) * 2 * nj, ctx->stream));
+        CUDA_TRY(ctx, cudaMemsetAsync(ctx->counts.p, 0, sizeof(unsigned long long) * 3 * nj, ctx->stream));
         if (timed) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_a, ctx->stream));
         launch_jobs_init(djobs, nj, ctx->stream);
         launch_init_slab0(djobs, nj, nmp, (int)std::min(max_slab, (size_t)INT32_MAX), ctx->stream);
@@ -497,8 +506,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             int rc = hook->after_batch(ctx, ids, djobs);
             if (rc) return rc;
         }
-        hcounts.resize(2 * nj);
-        CUDA_TRY(ctx, d2h(ctx, hcounts.data(), ctx->counts.p, sizeof(unsigned long long) * 2 * nj));
+        hcounts.resize(3 * nj);
+        CUDA_TRY(ctx, d2h(ctx, hcounts.data(), ctx->counts.p, sizeof(unsigned long long) * 3 * nj));
         if (early_exit)
             CUDA_TRY(ctx, d2h(ctx, jl_host.data(), jl_dev, sizeof(int32_t) * n_chains));
         CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
@@ -508,6 +517,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             for (int i = 0; i < nj; i++) {
                 ctx->last_cell_updates += (int64_t)hcounts[i];
                 ctx->last_effective += (int64_t)hcounts[nj + i];
+                ctx->last_useful += (int64_t)hcounts[2 * nj + i];
             }
         }
         if (timed) {

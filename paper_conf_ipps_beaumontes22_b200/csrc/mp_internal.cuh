@@ -46,6 +46,8 @@ struct Job {
     int32_t *kmin_l;    // window start of layer l for this job (written by trans_kernel)
     int32_t code_cap;   // row capacity of codes (>= longest window of the batch)
     int32_t pad_;
+    uint32_t *rowflag;  // [(L+1)][n_v]: 1 if row (l, v) holds a finite value (persist path)
+    unsigned long long *useful;  // live relaxations whose source row is not all +inf
 };
 
 // Result of a traceback, written by traceback_kernel.

@@ -104,6 +104,9 @@ void launch_jobs_init(Job *jobs, int n_jobs, cudaStream_t s) {
 __global__ void init_slab0_kernel(const Job *jobs, int nmp) {
     const Job &J = jobs[blockIdx.y];
     const int64_t cells = (int64_t)J.n_v * J.P * nmp;
+    if (J.rowflag)
+        for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < J.n_v; v += gridDim.x * blockDim.x)
+            J.rowflag[v] = 1u;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cells;
          i += (int64_t)gridDim.x * blockDim.x) {
         const int m = (int)(i % nmp);
@@ -264,21 +267,36 @@ __global__ void trans_kernel(const Job *jobs, int l) {
     const int v0 = blockIdx.x * 8;
     if (v0 >= J.n_v) return;
     const int vc = min(8, J.n_v - v0);
+    // the step kernel of layer l sets the row flags of slab l; clear them first
+    if (J.rowflag && threadIdx.x < vc) J.rowflag[(size_t)l * J.n_v + v0 + threadIdx.x] = 0u;
     const int kmin = max(kmin_of(J, l), kmin_mem(J, l));
     const int wl = l + 1 - kmin;   // may be <= 0
     if (blockIdx.x == 0 && threadIdx.x == 0) *J.kmin_l = kmin;
     const double Ul = J.Up[l];
-    unsigned live = 0;
+    unsigned live = 0, useful = 0;
     for (int e = threadIdx.x; e < vc * max(wl, 0); e += blockDim.x) {
         const int vv = e / wl, kk = e - vv * wl;
         const int k = kmin + kk;
-        const int32_t tr = transition(J, k, l, v0 + vv, __dsub_rn(Ul, J.Up[k - 1]), nullptr);
+        int32_t tr = transition(J, k, l, v0 + vv, __dsub_rn(Ul, J.Up[k - 1]), nullptr);
+        if (tr >= 0) {
+            live++;
+            // a source row that is +inf everywhere can only contribute +inf (exact skip)
+            if (J.rowflag && J.rowflag[(size_t)(k - 1) * J.n_v + (tr & 0xFFFF)] == 0u)
+                tr = (int32_t)0x80000001;
+            else
+                useful++;
+        }
         J.codes[(size_t)(v0 + vv) * J.code_cap + kk] = tr;
-        live += tr >= 0;
     }
-    for (int o = 16; o > 0; o >>= 1) live += __shfl_xor_sync(0xffffffffu, live, o);
-    if ((threadIdx.x & 31) == 0 && live && J.P > 1)
-        atomicAdd(J.eff, (unsigned long long)live * (unsigned long long)(J.P - 1) * (unsigned long long)J.n_m);
+    for (int o = 16; o > 0; o >>= 1) {
+        live += __shfl_xor_sync(0xffffffffu, live, o);
+        useful += __shfl_xor_sync(0xffffffffu, useful, o);
+    }
+    if ((threadIdx.x & 31) == 0 && live && J.P > 1) {
+        const unsigned long long per = (unsigned long long)(J.P - 1) * (unsigned long long)J.n_m;
+        atomicAdd(J.eff, (unsigned long long)live * per);
+        if (useful && J.useful) atomicAdd(J.useful, (unsigned long long)useful * per);
+    }
 }
 
 void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, cudaStream_t s) {

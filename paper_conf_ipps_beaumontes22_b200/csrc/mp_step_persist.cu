@@ -78,6 +78,7 @@ struct StageMeta {
     double tau;
     double U;                 // U(k,l) of the stage's k
     int32_t tr[kMaxVb];       // transition code per delay row (<0: not live)
+    uint32_t *flag;           // row flags of (l, v0): row v0+vv at flag[vv]
     int32_t rowlen;           // P*NMP
     int16_t np, vcount, n_m, flags;   // flags: 1 = last stage of the tile, 2 = no data, 4 = terminate
 };
@@ -144,6 +145,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
 #pragma unroll
                 for (int m = 0; m < NMP; m++)
                     o[m] = (m < n_m && U1l <= tau && (int64_t)m + d <= (int64_t)(n_m - 1)) ? U1l : MP_INF;
+                if (U1l <= tau && d <= (int64_t)(n_m - 1)) atomicOr(J.rowflag + (size_t)l * J.n_v + v, 1u);
             }
             if (np <= 0) continue;
             const int kmin = *J.kmin_l;
@@ -152,8 +154,9 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             const unsigned grp_mask = ((1u << vcount) - 1u) << (kk * vcount);
             const int32_t *codes = J.codes + (size_t)(v0 + v2) * J.code_cap;
             double *tile_out = out + (size_t)v0 * rowlen + (size_t)p_lo * NMP;
+            uint32_t *tile_flag = J.rowflag + (size_t)l * J.n_v + v0;
             auto fill_meta = [&](StageMeta &M, int flags) {
-                M.out = tile_out; M.tau = tau; M.rowlen = (int32_t)rowlen;
+                M.out = tile_out; M.tau = tau; M.rowlen = (int32_t)rowlen; M.flag = tile_flag;
                 M.np = (int16_t)np; M.vcount = (int16_t)vcount; M.n_m = (int16_t)n_m;
                 M.flags = (int16_t)flags;
             };
@@ -331,6 +334,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             if (active) {
                 const double tau = M.tau;
                 double *o = M.out + (size_t)vv * M.rowlen + (size_t)pp_off * NMP;
+                bool fin = false;
                 if (ROW) {
 #pragma unroll
                     for (int c = 0; c < C; c++) {
@@ -338,14 +342,17 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                         double2 r;
                         r.x = (2 * j < n_m && best[2 * c] <= tau) ? best[2 * c] : MP_INF;
                         r.y = (2 * j + 1 < n_m && best[2 * c + 1] <= tau) ? best[2 * c + 1] : MP_INF;
+                        fin |= (r.x <= tau) | (r.y <= tau);
                         *reinterpret_cast<double2 *>(o + 2 * j) = r;
                     }
                 } else {
                     double2 r;
                     r.x = (2 * h < n_m && best[0] <= tau) ? best[0] : MP_INF;
                     r.y = (2 * h + 1 < n_m && best[1] <= tau) ? best[1] : MP_INF;
+                    fin = (r.x <= tau) | (r.y <= tau);
                     *reinterpret_cast<double2 *>(o + 2 * h) = r;
                 }
+                if (fin) atomicOr(M.flag + vv, 1u);
             }
 #pragma unroll
             for (int i = 0; i < NB; i++) best[i] = MP_INF;
