@@ -97,6 +97,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
     __shared__ Job pJ;                               // producer's copy of the current tile's job
     __shared__ int32_t p_tr[kMaxGroups * kMaxVb];    // live codes of the round's groups
     __shared__ int32_t p_grp[kMaxGroups];            // k of each group
+    __shared__ double p_U[kMaxGroups];               // U(k,l) of each group
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
@@ -114,11 +115,17 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
 
     if (warp == kPCons / 32) {
         // ======================================================= producer warp
-        int gi = 0;
+        int gi = 0;              // stages issued so far
+        int slot0 = 0, use0 = 0; // slot of stage gi and how many times that slot was used before
         for (int tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
             const int jid = tile_job[tile];
             __syncwarp();
-            if (lane == 0) pJ = jobs[jid];
+            {   // cooperative copy of the job descriptor (one 8-byte word per lane)
+                static_assert(sizeof(Job) % 8 == 0 && sizeof(Job) <= 32 * 8 * 2, "Job size");
+                const uint64_t *src = reinterpret_cast<const uint64_t *>(jobs + jid);
+                uint64_t *dst = reinterpret_cast<uint64_t *>(&pJ);
+                for (int w = lane; w < (int)(sizeof(Job) / 8); w += 32) dst[w] = __ldg(src + w);
+            }
             __syncwarp();
             const Job &J = pJ;
             if (l > J.L) continue;
@@ -168,6 +175,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                     const int k = kb + kk;
                     const bool valid = kk < per && k <= l;
                     const int32_t tr = valid ? __ldg(codes + (k - kmin)) : -1;
+                    const double Ukl = (valid && v2 == 0) ? __dsub_rn(Ul, __ldg(J.Up + k - 1)) : 0.0;
                     const unsigned live = __ballot_sync(0xffffffffu, tr >= 0);
                     const bool leader = valid && (v2 == 0) && (live & grp_mask);
                     const unsigned leaders = __ballot_sync(0xffffffffu, leader);
@@ -175,7 +183,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                     const int myrank = __shfl_sync(0xffffffffu, rank, valid ? kk * vcount : 0);
                     if (valid && (live & grp_mask)) {
                         p_tr[myrank * kMaxVb + v2] = tr;
-                        if (v2 == 0) p_grp[myrank] = k;
+                        if (v2 == 0) { p_grp[myrank] = k; p_U[myrank] = Ukl; }
                     }
                     ngrp += __popc(leaders);
                 }
@@ -187,16 +195,16 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                 for (int g0 = 0; g0 < ngrp; g0 += nst) {
                     const int g = g0 + lane;
                     if (lane < nst && g < ngrp) {
-                        const int gg = gi + g;
-                        const int s = gg % nst;
-                        if (gg >= nst) mbar_wait(empty0 + 8 * s, (uint32_t)((gg / nst - 1) & 1));
-                        StageMeta &M = meta[s];
-                        fill_meta(M, done && g == ngrp - 1 ? 1 : 0);
+                        // stage gi+g -> slot and use count, without runtime division: the
+                        // round holds < nst stages, so the slot wraps at most once
+                        int s = slot0 + lane, use = use0;
+                        if (s >= nst) { s -= nst; use++; }
+                        if (use > 0) mbar_wait(empty0 + 8 * s, (uint32_t)((use - 1) & 1));
                         const int k = p_grp[g];
-                        M.U = __dsub_rn(Ul, J.Up[k - 1]);
                         const double *src = J.table + (size_t)(k - 1) * slab + (size_t)(p_lo - 1) * NMP;
                         uint32_t bytes = 0;
-                        for (int w = 0; w < kMaxVb; w++) {
+                        StageMeta &M = meta[s];
+                        for (int w = 0; w < kMaxVb; w++) {   // copies first, metadata after
                             const int32_t trw = w < vcount ? p_tr[g * kMaxVb + w] : -1;
                             M.tr[w] = trw;
                             if (trw < 0) continue;
@@ -204,29 +212,33 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                             bulk_g2s(ring_s + 8u * (uint32_t)(s * stage_doubles + w * seg_doubles),
                                      src + (size_t)(trw & 0xFFFF) * rowlen, seg_bytes, full0 + 8 * s);
                         }
+                        fill_meta(M, done && g == ngrp - 1 ? 1 : 0);
+                        M.U = p_U[g];
                         mbar_arrive_expect_tx(full0 + 8 * s, bytes);
                     }
                     __syncwarp();
+                    const int adv = min(nst, ngrp - g0);   // stages issued in this round
+                    slot0 += adv;
+                    if (slot0 >= nst) { slot0 -= nst; use0++; }
                 }
                 gi += ngrp;
                 if (done) { closed = ngrp > 0; break; }
             }
             if (!closed) {   // no live stage at the end of the window: close with an empty stage
                 if (lane == 0) {
-                    const int s = gi % nst;
-                    if (gi >= nst) mbar_wait(empty0 + 8 * s, (uint32_t)((gi / nst - 1) & 1));
-                    fill_meta(meta[s], 1 | 2);
-                    mbar_arrive(full0 + 8 * s);
+                    if (use0 > 0) mbar_wait(empty0 + 8 * slot0, (uint32_t)((use0 - 1) & 1));
+                    fill_meta(meta[slot0], 1 | 2);
+                    mbar_arrive(full0 + 8 * slot0);
                 }
                 gi += 1;
+                if (++slot0 == nst) { slot0 = 0; use0++; }
             }
         }
         __syncwarp();
         if (lane == 0) {
-            const int s = gi % nst;
-            if (gi >= nst) mbar_wait(empty0 + 8 * s, (uint32_t)((gi / nst - 1) & 1));
-            meta[s].flags = 4;
-            mbar_arrive(full0 + 8 * s);
+            if (use0 > 0) mbar_wait(empty0 + 8 * slot0, (uint32_t)((use0 - 1) & 1));
+            meta[slot0].flags = 4;
+            mbar_arrive(full0 + 8 * slot0);
         }
         return;
     }
@@ -238,9 +250,9 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
     for (int i = 0; i < NB; i++) best[i] = MP_INF;
     int cur_np = -1, cur_vc = -1, vv = 0, pp_off = 0, h = 0, rot = 0;
     bool active = false;
-    for (int gi = 0;; gi++) {
-        const int s = gi % nst;
-        mbar_wait(full0 + 8 * s, (uint32_t)((gi / nst) & 1));
+    int s = 0, phase = 0;
+    for (;; ) {
+        mbar_wait(full0 + 8 * s, (uint32_t)phase);
         const StageMeta &M = meta[s];
         const int flags = M.flags;
         if (flags & 4) break;
@@ -359,6 +371,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(empty0 + 8 * s);
+        if (++s == nst) { s = 0; phase ^= 1; }
     }
 }
 
