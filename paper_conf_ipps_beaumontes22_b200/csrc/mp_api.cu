@@ -396,6 +396,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             const ChainSpec &c = cs[s.chain];
             const size_t bytes = table_doubles(c, disc) * 8;
             if (!hjobs.empty() && (used + bytes > budget || hjobs.size() >= cap_jobs)) break;
+            // the persistent step kernel needs one tile geometry per launch: uniform P
+            if (ctx->kernel == 2 && !hjobs.empty() && c.P != hjobs[0].P) break;
             if (hjobs.empty() && bytes > budget && bytes > ctx->tables.n) {
                 // a single job larger than the budget: try anyway (may fail with ENOMEM)
             }
@@ -410,7 +412,6 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             int n_tiles;
             if (ctx->kernel == 2) {
                 persist_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
-                stage_doubles = std::max(stage_doubles, J.vb * (J.np + 1) * nmp);
             } else if (ctx->kernel == 1) {
                 tma_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
                 smem_tma = std::max(smem_tma, tma_smem_bytes(J.vb, J.np, nmp));
@@ -467,11 +468,13 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         launch_init_slab0(djobs, nj, nmp, (int)std::min(max_slab, (size_t)INT32_MAX), ctx->stream);
         ctx->launches += 2;
         const int n_tiles = (int)htiles.size();
-        int persist_grid = 0, nst = 0;
+        int persist_grid = 0, nsg = 0, p_np = 0, p_vb = 0;
         if (ctx->kernel == 2) {
-            nst = persist_nst(stage_doubles);
-            if (nst < 2) return fail(ctx, MADPIPE_EINVAL, "row segment too large for the step kernel ring");
-            persist_grid = std::min(n_tiles, ctx->num_sms * persist_blocks_per_sm(nmp, stage_doubles, nst));
+            p_np = hjobs[0].np;
+            p_vb = hjobs[0].vb;
+            nsg = persist_nsg(p_np, p_vb, nmp);
+            if (nsg < 2) return fail(ctx, MADPIPE_EINVAL, "row segment too large for the step kernel ring");
+            persist_grid = std::min(n_tiles, ctx->num_sms * persist_blocks_per_sm(nmp, p_np, p_vb, nsg));
         }
         const bool per_launch = timed && ctx->per_launch_timing;
         if (per_launch && ctx->ev_pool.size() < (size_t)(2 * maxL)) {
@@ -488,7 +491,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 ctx->launches++;
             }
             if (ctx->kernel == 2)
-                launch_step_persist(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, stage_doubles, nst,
+                launch_step_persist(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, p_np, p_vb, nsg,
                                     persist_grid, ctx->stream);
             else if (ctx->kernel == 1)
                 launch_step_tma(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, smem_tma, ctx->stream);
@@ -778,6 +781,10 @@ extern "C" int madpipe_solve_batch(madpipe_ctx *ctx, int32_t n, const madpipe_ch
     std::vector<JobSpec> js;
     for (int j = 0; j < disc->n_periods; j++)
         for (int c = 0; c < n; c++) js.push_back({c, j});
+    // group by P (the persistent step kernel launches one tile geometry at a time);
+    // within a group the order stays candidate-major
+    std::stable_sort(js.begin(), js.end(),
+                     [&](const JobSpec &a, const JobSpec &b) { return cs[a.chain].P < cs[b.chain].P; });
     std::vector<uint64_t> counts;
     rc = run_jobs(ctx, cs, cd, disc, js, (int32_t *)ctx->jl.p, nullptr, nullptr, &counts,
                   disc->early_exit != 0, nullptr, true);

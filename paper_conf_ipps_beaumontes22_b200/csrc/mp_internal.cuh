@@ -79,11 +79,11 @@ void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, i
 void launch_step_tma(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int smem,
                      cudaStream_t s);
 int tma_smem_bytes(int vb, int np, int nmp);
-void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp,
-                         int stage_doubles, int nst, int grid, cudaStream_t s);
-int persist_blocks_per_sm(int nmp, int stage_doubles, int nst);
+void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np,
+                         int vb, int nsg, int grid, cudaStream_t s);
+int persist_blocks_per_sm(int nmp, int np, int vb, int nsg);
 void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
-int persist_nst(int stage_doubles);
+int persist_nsg(int np, int vb, int nmp);
 void tma_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
 void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, cudaStream_t s);
 void launch_root(const Job *jobs, int n_jobs, int nmp, int32_t *jl_per_chain, double *root_out,

@@ -6,23 +6,29 @@
 //        N: A[k-1][v'][p-1][m]            (normal GPU fits)
 //        S: U(k,l) + A[k-1][v'][p][m+d]   (special GPU) ).
 // The transitions (k, v) -> (v', nf, d) of layer l were computed beforehand by
-// trans_kernel (a3) into J.codes, for the window starting at *J.kmin_l.
+// trans_kernel (a3) into J.codes for the window starting at *J.kmin_l; a
+// transition whose source row is +inf everywhere is already marked dead there.
 //
 // Structure:
-//   * grid = resident CTAs (1-2 per SM); CTA c takes tiles c, c+G, c+2G, ...
-//     A tile is vb delay rows x np processor rows of one job.
+//   * grid = resident CTAs (2 per SM); CTA c takes tiles c, c+G, c+2G, ...  A
+//     tile is vb delay rows x np processor rows of one job; every job of a launch
+//     has the same P, hence the same tile geometry (passed as arguments).
+//   * per-row sub-rings: delay row w of a tile owns a ring of nsg one-row slots in
+//     shared memory, with its own full/empty mbarriers, consumed by its own warp
+//     group.  Every slot carries exactly one useful source row segment, so the
+//     bytes in flight per SM stay at the ring capacity whatever the liveness.
 //   * warp 8 is the producer.  Per tile it writes the base row p = 0 (a4),
-//     reads the window's codes (32 at a time, one coalesced load per lane),
-//     compacts the k with a live row (ballot), and for each such k streams the
-//     source row segments A[k-1][v'][p_lo-1 .. p_lo+np-1][*] of the live delay
-//     rows into a `nst`-stage shared-memory ring with cp.async.bulk, each stage
-//     completing on its mbarrier.  Up to nst lanes issue stages concurrently.
-//   * warps 0-7 are consumers.  ROW mode (NMP <= 16): a thread owns one
-//     (v, p) row of NMP levels as NMP/2 16-byte chunks held in a lane-rotated
-//     order, which makes every quarter-warp's 16-byte shared loads hit 8
-//     distinct bank groups while register indices stay compile-time.  PAIR mode
-//     (NMP >= 32): a thread owns one (v, p, m-pair).  Either way the shift d is
-//     uniform per warp.  At the tile's last stage they clamp to tau and store.
+//     reads the window's codes 32 at a time (one coalesced load per lane), builds
+//     per-row lists of live k with ballots, and then issues, lane-parallel across
+//     rows and stages, one cp.async.bulk per live (k, row): the segment
+//     A[k-1][v'][p_lo-1 .. p_lo+np-1][*] into the row's next slot, completing on
+//     the slot's mbarrier.
+//   * warps 0-7 are consumers, one group per delay row.  ROW mode (NMP <= 16):
+//     a thread owns one (v, p) row of NMP levels as NMP/2 16-byte chunks held in
+//     a lane-rotated order (every quarter-warp's 16-byte shared loads hit 8
+//     distinct bank groups; register indices stay compile-time).  PAIR mode
+//     (NMP >= 32): a thread owns one (v, p, m-pair).  At the row's last stage
+//     the group clamps to tau, stores, and flags the row finite/infinite.
 // min is exact and order-free, so results equal the oracle's bit for bit.
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -67,47 +73,53 @@ __device__ __forceinline__ double dmin(double a, double b) { return b < a ? b : 
 
 }  // namespace
 
-constexpr int kNstMax = 12;          // ring stages (runtime nst <= kNstMax)
+constexpr int kSlotsMax = 64;        // one-row slots per CTA (all rings)
 constexpr int kPCons = 256;          // consumer threads (8 warps); + 1 producer warp
-constexpr int kMaxVb = 8;            // delay rows per tile
-constexpr int kMaxGroups = 128;      // live k collected per producer round
+constexpr int kMaxVb = 8;            // delay rows (= rings) per tile
+constexpr int kSpan = 128;           // k per producer chunk
 
-// per-stage metadata written by the producer, read by the consumers
-struct StageMeta {
-    double *out;              // output of row v0, processor p_lo (row v0+vv at out + vv*rowlen)
+struct SlotMeta {
+    double *out;        // output row segment: A[l][v][p_lo][0]
+    uint32_t *flag;     // row flag of (l, v)
     double tau;
-    double U;                 // U(k,l) of the stage's k
-    int32_t tr[kMaxVb];       // transition code per delay row (<0: not live)
-    uint32_t *flag;           // row flags of (l, v0): row v0+vv at flag[vv]
-    int32_t rowlen;           // P*NMP
-    int16_t np, vcount, n_m, flags;   // flags: 1 = last stage of the tile, 2 = no data, 4 = terminate
+    double U;           // U(k,l)
+    int32_t tr;         // transition code
+    int32_t np;         // processor rows of the tile (<= np_max)
+    int16_t n_m, flags; // flags: 1 = last stage of the row, 2 = no data, 4 = terminate
+    int32_t pad_;
 };
 
 template <int NMP>
 __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job *__restrict__ jobs,
                                                                       const int32_t *__restrict__ tile_job,
-                                                                      int n_tiles, int l, int stage_doubles,
-                                                                      int nst) {
+                                                                      int n_tiles, int l, int np_max, int vb,
+                                                                      int nsg) {
     constexpr int C = NMP / 2;                       // 16-byte chunks per processor row
     constexpr bool ROW = NMP <= 16;
+    constexpr int PER_ROW = ROW ? 1 : C;             // consumer threads per processor row
     extern __shared__ __align__(128) unsigned char dsm[];
-    __shared__ __align__(8) uint64_t full[kNstMax];
-    __shared__ __align__(8) uint64_t empty[kNstMax];
-    __shared__ StageMeta meta[kNstMax];
+    __shared__ __align__(8) uint64_t full[kSlotsMax];
+    __shared__ __align__(8) uint64_t empty[kSlotsMax];
+    __shared__ SlotMeta meta[kSlotsMax];
     __shared__ Job pJ;                               // producer's copy of the current tile's job
-    __shared__ int32_t p_tr[kMaxGroups * kMaxVb];    // live codes of the round's groups
-    __shared__ int32_t p_grp[kMaxGroups];            // k of each group
-    __shared__ double p_U[kMaxGroups];               // U(k,l) of each group
+    __shared__ int16_t p_k[kMaxVb][kSpan];           // live k (offset in the chunk) per row
+    __shared__ int32_t p_code[kMaxVb][kSpan];        // its transition code
+    __shared__ double p_Uk[kSpan];                   // U(k,l) per k of the chunk
+    __shared__ int p_sl[kMaxVb], p_us[kMaxVb];       // per ring: next slot, its use count
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
+    const int rowgroup = ((np_max * PER_ROW + 31) / 32) * 32;   // threads per ring group
+    const int wpg = rowgroup / 32;                               // warps per ring group
+    const int seg_doubles = (np_max + 1) * NMP;                  // slot size
     const uint32_t full0 = smem_u32(&full[0]), empty0 = smem_u32(&empty[0]);
     const uint32_t ring_s = smem_u32(dsm);
     if (tid == 0) {
-        for (int s = 0; s < nst; s++) {
+        for (int s = 0; s < vb * nsg; s++) {
             mbar_init(full0 + 8 * s, 1);
-            mbar_init(empty0 + 8 * s, kPCons / 32);
+            mbar_init(empty0 + 8 * s, wpg);
         }
+        for (int w = 0; w < kMaxVb; w++) { p_sl[w] = 0; p_us[w] = 0; }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -115,8 +127,9 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
 
     if (warp == kPCons / 32) {
         // ======================================================= producer warp
-        int gi = 0;              // stages issued so far
-        int slot0 = 0, use0 = 0; // slot of stage gi and how many times that slot was used before
+        const int lpr = 32 / vb;                     // lanes per ring in the issue phase
+        const int m_round = min(nsg, lpr);           // stages per ring per issue round
+        const int iw = lane / lpr, ij = lane - (lane / lpr) * lpr;
         for (int tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
             const int jid = tile_job[tile];
             __syncwarp();
@@ -137,8 +150,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             const int np = max(0, min(J.np, J.P - p_lo));
             const size_t rowlen = (size_t)J.P * NMP;
             const size_t slab = (size_t)J.n_v * rowlen;
-            const int seg_doubles = (np + 1) * NMP;
-            const uint32_t seg_bytes = (uint32_t)seg_doubles * 8u;
+            const uint32_t seg_bytes = (uint32_t)(np + 1) * NMP * 8u;
             double *out = J.table + (size_t)l * slab;
             const double Ul = J.Up[l];
             const double tau = J.tau;
@@ -158,195 +170,183 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             const int kmin = *J.kmin_l;
             const int per = 32 / vcount;              // k per pass (vcount <= 8)
             const int kk = lane / vcount, v2 = lane - kk * vcount;
-            const unsigned grp_mask = ((1u << vcount) - 1u) << (kk * vcount);
+            unsigned rowmask = 0;                     // lanes holding my row v2
+            for (int q = 0; q < per; q++) rowmask |= 1u << (q * vcount + v2);
             const int32_t *codes = J.codes + (size_t)(v0 + v2) * J.code_cap;
-            double *tile_out = out + (size_t)v0 * rowlen + (size_t)p_lo * NMP;
-            uint32_t *tile_flag = J.rowflag + (size_t)l * J.n_v + v0;
-            auto fill_meta = [&](StageMeta &M, int flags) {
-                M.out = tile_out; M.tau = tau; M.rowlen = (int32_t)rowlen; M.flag = tile_flag;
-                M.np = (int16_t)np; M.vcount = (int16_t)vcount; M.n_m = (int16_t)n_m;
-                M.flags = (int16_t)flags;
-            };
-            bool closed = false;
-            for (int kb = kmin; kb <= l;) {
-                // ---- collect up to kMaxGroups live groups (k with >= 1 live delay row)
-                int ngrp = 0;
-                for (; kb <= l && ngrp + per <= kMaxGroups; kb += per) {
+            for (int kc0 = kmin; kc0 <= l; kc0 += kSpan) {
+                const int kc1 = min(l + 1, kc0 + kSpan);
+                const bool done = kc1 > l;
+                // ---- per-row lists of live k in [kc0, kc1)
+                int cnt = 0;                          // live entries of row v2 so far (per lane)
+                for (int kb = kc0; kb < kc1; kb += per) {
                     const int k = kb + kk;
-                    const bool valid = kk < per && k <= l;
+                    const bool valid = kk < per && k < kc1;
                     const int32_t tr = valid ? __ldg(codes + (k - kmin)) : -1;
-                    const double Ukl = (valid && v2 == 0) ? __dsub_rn(Ul, __ldg(J.Up + k - 1)) : 0.0;
-                    const unsigned live = __ballot_sync(0xffffffffu, tr >= 0);
-                    const bool leader = valid && (v2 == 0) && (live & grp_mask);
-                    const unsigned leaders = __ballot_sync(0xffffffffu, leader);
-                    const int rank = ngrp + __popc(leaders & ((1u << lane) - 1u));
-                    const int myrank = __shfl_sync(0xffffffffu, rank, valid ? kk * vcount : 0);
-                    if (valid && (live & grp_mask)) {
-                        p_tr[myrank * kMaxVb + v2] = tr;
-                        if (v2 == 0) { p_grp[myrank] = k; p_U[myrank] = Ukl; }
+                    if (valid && v2 == 0) p_Uk[k - kc0] = __dsub_rn(Ul, __ldg(J.Up + k - 1));
+                    const unsigned live = __ballot_sync(0xffffffffu, tr >= 0) & (valid ? 0xffffffffu : 0u);
+                    const unsigned mine = __ballot_sync(0xffffffffu, tr >= 0) & rowmask;
+                    if (tr >= 0) {
+                        const int pos = cnt + __popc(mine & ((1u << lane) - 1u));
+                        p_k[v2][pos] = (int16_t)(k - kc0);
+                        p_code[v2][pos] = tr;
                     }
-                    ngrp += __popc(leaders);
+                    (void)live;
+                    cnt += __popc(mine);
                 }
-                const bool done = kb > l;
                 __syncwarp();
-                // ---- one stage per live group, in rounds of at most nst stages: the slots
-                // of a round are distinct, so each lane's parity wait refers to the previous
-                // use of its own slot (never two phases ahead, where mbarrier parity aliases)
-                for (int g0 = 0; g0 < ngrp; g0 += nst) {
-                    const int g = g0 + lane;
-                    if (lane < nst && g < ngrp) {
-                        // stage gi+g -> slot and use count, without runtime division: the
-                        // round holds < nst stages, so the slot wraps at most once
-                        int s = slot0 + lane, use = use0;
-                        if (s >= nst) { s -= nst; use++; }
-                        if (use > 0) mbar_wait(empty0 + 8 * s, (uint32_t)((use - 1) & 1));
-                        const int k = p_grp[g];
-                        const double *src = J.table + (size_t)(k - 1) * slab + (size_t)(p_lo - 1) * NMP;
-                        uint32_t bytes = 0;
-                        StageMeta &M = meta[s];
-                        for (int w = 0; w < kMaxVb; w++) {   // copies first, metadata after
-                            const int32_t trw = w < vcount ? p_tr[g * kMaxVb + w] : -1;
-                            M.tr[w] = trw;
-                            if (trw < 0) continue;
-                            bytes += seg_bytes;
-                            bulk_g2s(ring_s + 8u * (uint32_t)(s * stage_doubles + w * seg_doubles),
-                                     src + (size_t)(trw & 0xFFFF) * rowlen, seg_bytes, full0 + 8 * s);
+                // ---- issue: lane (iw, ij) takes stages ij, ij+m, ... of ring iw
+                const int n_w = __shfl_sync(0xffffffffu, cnt, iw < vcount ? iw : 0);
+                const bool my_ring = iw < vcount;
+                const int n_eff = my_ring ? (n_w > 0 ? n_w : (done ? 1 : 0)) : 0;   // 1 = closing stage
+                int max_n = n_eff;
+                for (int o = 16; o > 0; o >>= 1) max_n = max(max_n, __shfl_xor_sync(0xffffffffu, max_n, o));
+                for (int r0 = 0; r0 < max_n; r0 += m_round) {
+                    const int q = r0 + ij;
+                    if (my_ring && ij < m_round && q < n_eff) {
+                        int s = p_sl[iw] + ij, use = p_us[iw];
+                        if (s >= nsg) { s -= nsg; use++; }
+                        const int slot = iw * nsg + s;
+                        if (use > 0) mbar_wait(empty0 + 8 * slot, (uint32_t)((use - 1) & 1));
+                        SlotMeta &M = meta[slot];
+                        M.out = out + (size_t)(v0 + iw) * rowlen + (size_t)p_lo * NMP;
+                        M.flag = J.rowflag + (size_t)l * J.n_v + v0 + iw;
+                        M.tau = tau;
+                        M.np = np;
+                        M.n_m = (int16_t)n_m;
+                        if (n_w == 0) {              // closing stage without data
+                            M.flags = 1 | 2;
+                            M.tr = -1;
+                            mbar_arrive(full0 + 8 * slot);
+                        } else {
+                            const int kofs = p_k[iw][q];
+                            const int32_t tr = p_code[iw][q];
+                            const int k = kc0 + kofs;
+                            bulk_g2s(ring_s + 8u * (uint32_t)(slot * seg_doubles),
+                                     J.table + (size_t)(k - 1) * slab + (size_t)(tr & 0xFFFF) * rowlen +
+                                         (size_t)(p_lo - 1) * NMP,
+                                     seg_bytes, full0 + 8 * slot);
+                            M.flags = (int16_t)(done && q == n_w - 1 ? 1 : 0);
+                            M.tr = tr;
+                            M.U = p_Uk[kofs];
+                            mbar_arrive_expect_tx(full0 + 8 * slot, seg_bytes);
                         }
-                        fill_meta(M, done && g == ngrp - 1 ? 1 : 0);
-                        M.U = p_U[g];
-                        mbar_arrive_expect_tx(full0 + 8 * s, bytes);
                     }
                     __syncwarp();
-                    const int adv = min(nst, ngrp - g0);   // stages issued in this round
-                    slot0 += adv;
-                    if (slot0 >= nst) { slot0 -= nst; use0++; }
+                    if (my_ring && ij == 0) {         // advance ring iw by the stages of this round
+                        const int adv = max(0, min(m_round, n_eff - r0));
+                        int s = p_sl[iw] + adv;
+                        if (s >= nsg) { s -= nsg; p_us[iw]++; }
+                        p_sl[iw] = s;
+                    }
+                    __syncwarp();
                 }
-                gi += ngrp;
-                if (done) { closed = ngrp > 0; break; }
-            }
-            if (!closed) {   // no live stage at the end of the window: close with an empty stage
-                if (lane == 0) {
-                    if (use0 > 0) mbar_wait(empty0 + 8 * slot0, (uint32_t)((use0 - 1) & 1));
-                    fill_meta(meta[slot0], 1 | 2);
-                    mbar_arrive(full0 + 8 * slot0);
-                }
-                gi += 1;
-                if (++slot0 == nst) { slot0 = 0; use0++; }
+                if (done) break;
             }
         }
         __syncwarp();
-        if (lane == 0) {
-            if (use0 > 0) mbar_wait(empty0 + 8 * slot0, (uint32_t)((use0 - 1) & 1));
-            meta[slot0].flags = 4;
-            mbar_arrive(full0 + 8 * slot0);
+        if (lane < vb) {   // terminate every ring
+            const int w = lane;
+            const int slot = w * nsg + p_sl[w];
+            if (p_us[w] > 0) mbar_wait(empty0 + 8 * slot, (uint32_t)((p_us[w] - 1) & 1));
+            meta[slot].flags = 4;
+            mbar_arrive(full0 + 8 * slot);
         }
         return;
     }
 
     // =========================================================== consumer warps
-    constexpr int NB = ROW ? NMP : 2;   // accumulators per thread
+    const int grp = warp / wpg;                      // my ring
+    if (grp >= vb) return;                           // idle warps (vb * wpg < 8)
+    const int q = tid - grp * rowgroup;
+    int pp_off, h = 0, rot = 0;
+    if (ROW) {
+        pp_off = q;
+        constexpr int G8 = C >= 8 ? 1 : 8 / C;       // lanes sharing a 128-byte window
+        constexpr int RM = C >= 8 ? 8 : C;
+        rot = (pp_off / G8) % RM;
+    } else {
+        pp_off = q / C;
+        h = q - pp_off * C;
+    }
+    constexpr int NB = ROW ? NMP : 2;                // accumulators per thread
     double best[NB];
 #pragma unroll
     for (int i = 0; i < NB; i++) best[i] = MP_INF;
-    int cur_np = -1, cur_vc = -1, vv = 0, pp_off = 0, h = 0, rot = 0;
-    bool active = false;
     int s = 0, phase = 0;
-    for (;; ) {
-        mbar_wait(full0 + 8 * s, (uint32_t)phase);
-        const StageMeta &M = meta[s];
+    for (;;) {
+        const int slot = grp * nsg + s;
+        mbar_wait(full0 + 8 * slot, (uint32_t)phase);
+        const SlotMeta &M = meta[slot];
         const int flags = M.flags;
         if (flags & 4) break;
-        const int np = M.np, vcount = M.vcount, n_m = M.n_m;
-        if (np != cur_np || vcount != cur_vc) {
-            if (ROW) {
-                const int rowgroup = ((np + 31) / 32) * 32;
-                vv = tid / rowgroup;
-                pp_off = tid - vv * rowgroup;
-                // lane rotation of the chunks: 8 consecutive threads of a quarter-warp
-                // start at 8 distinct 16-byte bank groups
-                constexpr int G8 = C >= 8 ? 1 : 8 / C;
-                constexpr int RM = C >= 8 ? 8 : C;
-                rot = (pp_off / G8) % RM;
-                active = vv < vcount && pp_off < np;
-            } else {
-                const int rowgroup = ((np * C + 31) / 32) * 32;
-                vv = tid / rowgroup;
-                const int q = tid - vv * rowgroup;
-                pp_off = q / C;
-                h = q - pp_off * C;
-                active = vv < vcount && pp_off < np;
-            }
-            cur_np = np; cur_vc = vcount;
-        }
+        const int np = M.np, n_m = M.n_m;
+        const bool active = pp_off < np;
         if (!(flags & 2) && active) {
-            const int32_t tr = M.tr[vv];
-            if (tr >= 0) {
-                const double *seg = ring + (size_t)s * stage_doubles + (size_t)vv * (np + 1) * NMP;
-                const double *rowN = seg + pp_off * NMP;           // processor p-1
-                const double *rowS = rowN + NMP;                    // processor p
-                const int d = (tr >> 16) & 0xFF;
-                const double U = M.U;
-                if (ROW) {
-                    if (tr & (1 << 24)) {                           // N
+            const int32_t tr = M.tr;
+            const double *rowN = ring + (size_t)slot * seg_doubles + pp_off * NMP;   // processor p-1
+            const double *rowS = rowN + NMP;                                          // processor p
+            const int d = (tr >> 16) & 0xFF;
+            const double U = M.U;
+            if (ROW) {
+                if (tr & (1 << 24)) {                           // N
+#pragma unroll
+                    for (int c = 0; c < C; c++) {
+                        const int j = (c + rot) & (C - 1);
+                        const double2 x = *reinterpret_cast<const double2 *>(rowN + 2 * j);
+                        best[2 * c] = dmin(best[2 * c], x.x);
+                        best[2 * c + 1] = dmin(best[2 * c + 1], x.y);
+                    }
+                }
+                if (d <= n_m - 1) {                             // S
+                    if ((d & 1) == 0) {
+                        const int e = d >> 1;
 #pragma unroll
                         for (int c = 0; c < C; c++) {
                             const int j = (c + rot) & (C - 1);
-                            const double2 x = *reinterpret_cast<const double2 *>(rowN + 2 * j);
-                            best[2 * c] = dmin(best[2 * c], x.x);
-                            best[2 * c + 1] = dmin(best[2 * c + 1], x.y);
-                        }
-                    }
-                    if (d <= n_m - 1) {                             // S
-                        if ((d & 1) == 0) {
-                            const int e = d >> 1;
-#pragma unroll
-                            for (int c = 0; c < C; c++) {
-                                const int j = (c + rot) & (C - 1);
-                                if (2 * j + d <= n_m - 1) {
-                                    const double2 y = *reinterpret_cast<const double2 *>(rowS + 2 * (j + e));
-                                    best[2 * c] = dmin(best[2 * c], __dadd_rn(U, y.x));
-                                    if (2 * j + 1 + d <= n_m - 1)
-                                        best[2 * c + 1] = dmin(best[2 * c + 1], __dadd_rn(U, y.y));
-                                }
-                            }
-                        } else {
-#pragma unroll
-                            for (int c = 0; c < C; c++) {
-                                const int j = (c + rot) & (C - 1);
-                                if (2 * j + d <= n_m - 1)
-                                    best[2 * c] = dmin(best[2 * c], __dadd_rn(U, rowS[2 * j + d]));
+                            if (2 * j + d <= n_m - 1) {
+                                const double2 y = *reinterpret_cast<const double2 *>(rowS + 2 * (j + e));
+                                best[2 * c] = dmin(best[2 * c], __dadd_rn(U, y.x));
                                 if (2 * j + 1 + d <= n_m - 1)
-                                    best[2 * c + 1] = dmin(best[2 * c + 1], __dadd_rn(U, rowS[2 * j + 1 + d]));
+                                    best[2 * c + 1] = dmin(best[2 * c + 1], __dadd_rn(U, y.y));
                             }
                         }
-                    }
-                } else {
-                    if (tr & (1 << 24)) {
-                        const double2 x = *reinterpret_cast<const double2 *>(rowN + 2 * h);
-                        best[0] = dmin(best[0], x.x);
-                        best[1] = dmin(best[1], x.y);
-                    }
-                    const int m0 = 2 * h + d;
-                    if (m0 <= n_m - 1) {
-                        double y0, y1;
-                        if ((d & 1) == 0) {
-                            const double2 y = *reinterpret_cast<const double2 *>(rowS + m0);
-                            y0 = y.x; y1 = y.y;
-                        } else {
-                            y0 = rowS[m0];
-                            y1 = (m0 + 1 <= n_m - 1) ? rowS[m0 + 1] : MP_INF;
+                    } else {
+#pragma unroll
+                        for (int c = 0; c < C; c++) {
+                            const int j = (c + rot) & (C - 1);
+                            if (2 * j + d <= n_m - 1)
+                                best[2 * c] = dmin(best[2 * c], __dadd_rn(U, rowS[2 * j + d]));
+                            if (2 * j + 1 + d <= n_m - 1)
+                                best[2 * c + 1] = dmin(best[2 * c + 1], __dadd_rn(U, rowS[2 * j + 1 + d]));
                         }
-                        best[0] = dmin(best[0], __dadd_rn(U, y0));
-                        if (m0 + 1 <= n_m - 1) best[1] = dmin(best[1], __dadd_rn(U, y1));
                     }
+                }
+            } else {
+                if (tr & (1 << 24)) {
+                    const double2 x = *reinterpret_cast<const double2 *>(rowN + 2 * h);
+                    best[0] = dmin(best[0], x.x);
+                    best[1] = dmin(best[1], x.y);
+                }
+                const int m0 = 2 * h + d;
+                if (m0 <= n_m - 1) {
+                    double y0, y1;
+                    if ((d & 1) == 0) {
+                        const double2 y = *reinterpret_cast<const double2 *>(rowS + m0);
+                        y0 = y.x; y1 = y.y;
+                    } else {
+                        y0 = rowS[m0];
+                        y1 = (m0 + 1 <= n_m - 1) ? rowS[m0 + 1] : MP_INF;
+                    }
+                    best[0] = dmin(best[0], __dadd_rn(U, y0));
+                    if (m0 + 1 <= n_m - 1) best[1] = dmin(best[1], __dadd_rn(U, y1));
                 }
             }
         }
-        if (flags & 1) {   // tile complete: clamp (Q12) and store
+        if (flags & 1) {   // row complete: clamp (Q12), store, flag
+            bool fin = false;
             if (active) {
                 const double tau = M.tau;
-                double *o = M.out + (size_t)vv * M.rowlen + (size_t)pp_off * NMP;
-                bool fin = false;
+                double *o = M.out + (size_t)pp_off * NMP;
                 if (ROW) {
 #pragma unroll
                     for (int c = 0; c < C; c++) {
@@ -364,14 +364,14 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                     fin = (r.x <= tau) | (r.y <= tau);
                     *reinterpret_cast<double2 *>(o + 2 * h) = r;
                 }
-                if (fin) atomicOr(M.flag + vv, 1u);
             }
+            if (__ballot_sync(0xffffffffu, fin) && lane == 0) atomicOr(M.flag, 1u);
 #pragma unroll
             for (int i = 0; i < NB; i++) best[i] = MP_INF;
         }
         __syncwarp();
-        if (lane == 0) mbar_arrive(empty0 + 8 * s);
-        if (++s == nst) { s = 0; phase ^= 1; }
+        if (lane == 0) mbar_arrive(empty0 + 8 * slot);
+        if (++s == nsg) { s = 0; phase ^= 1; }
     }
 }
 
@@ -392,29 +392,30 @@ void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int 
     *n_tiles = ((n_v + *vb - 1) / *vb) * *n_ptiles;
 }
 
-// ring depth that fits in ~100 KB of dynamic shared memory (2 CTAs per SM)
-int persist_nst(int stage_doubles) {
-    int n = (96 * 1024) / (stage_doubles * 8);
-    if (n > kNstMax) n = kNstMax;
-    return n;   // the caller falls back to another step kernel if n < 2
+// slots per ring: as many one-row slots as fit in ~96 KB, split over the vb rings
+int persist_nsg(int np, int vb, int nmp) {
+    const int seg = (np + 1) * nmp * 8;
+    int slots = (96 * 1024) / seg;
+    if (slots > kSlotsMax) slots = kSlotsMax;
+    return slots / vb;   // the caller falls back to another step kernel if < 2
 }
 
-void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp,
-                         int stage_doubles, int nst, int grid, cudaStream_t s) {
-    const int smem = nst * stage_doubles * 8;
+void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np,
+                         int vb, int nsg, int grid, cudaStream_t s) {
+    const int smem = vb * nsg * (np + 1) * nmp * 8;
     switch (nmp) {
 #define MP_CASE(N)                                                                                      \
     case N:                                                                                             \
         cudaFuncSetAttribute(step_persist_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
-        step_persist_kernel<N><<<grid, kPCons + 32, smem, s>>>(jobs, tile_job, n_tiles, l, stage_doubles, nst); \
+        step_persist_kernel<N><<<grid, kPCons + 32, smem, s>>>(jobs, tile_job, n_tiles, l, np, vb, nsg); \
         break;
         MP_CASE(2) MP_CASE(4) MP_CASE(8) MP_CASE(16) MP_CASE(32) MP_CASE(64)
 #undef MP_CASE
     }
 }
 
-int persist_blocks_per_sm(int nmp, int stage_doubles, int nst) {
-    const int smem = nst * stage_doubles * 8;
+int persist_blocks_per_sm(int nmp, int np, int vb, int nsg) {
+    const int smem = vb * nsg * (np + 1) * nmp * 8;
     int n = 0;
     switch (nmp) {
 #define MP_OCC(N)                                                                                       \
