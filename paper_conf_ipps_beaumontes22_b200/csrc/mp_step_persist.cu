@@ -173,7 +173,9 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             unsigned rowmask = 0;                     // lanes holding my row v2
             for (int q = 0; q < per; q++) rowmask |= 1u << (q * vcount + v2);
             const int32_t *codes = J.codes + (size_t)(v0 + v2) * J.code_cap;
-            for (int kc0 = kmin; kc0 <= l; kc0 += kSpan) {
+            // (kmin may be l+1: an empty window still runs one chunk, whose rows all get a
+            // closing stage, so every consumer group sees the end of every tile)
+            for (int kc0 = kmin;; kc0 += kSpan) {
                 const int kc1 = min(l + 1, kc0 + kSpan);
                 const bool done = kc1 > l;
                 // ---- per-row lists of live k in [kc0, kc1)
