@@ -51,6 +51,8 @@ struct madpipe_ctx {
     int64_t last_cell_updates = 0, last_effective = 0, last_useful = 0;
     int per_launch_timing = 0;
     int kernel = 2;           // MADPIPE_KERNEL: v1 = plain loads, tma = per-tile TMA, persist (default)
+    int prof = 0;             // MADPIPE_PROF=1: cycle counters of the persistent step kernel to stderr
+    DevBuf profbuf;
     int num_sms = 148;
     std::vector<cudaEvent_t> ev_pool;
 };
@@ -220,6 +222,8 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stre
     if (kern && strcmp(kern, "v1") == 0) c->kernel = 0;
     if (kern && strcmp(kern, "tma") == 0) c->kernel = 1;
     cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device);
+    const char *pf = getenv("MADPIPE_PROF");
+    c->prof = pf && pf[0] == '1';
     cudaEventCreate(&c->ev_a);
     cudaEventCreate(&c->ev_b);
     *out = c;
@@ -230,6 +234,7 @@ extern "C" void madpipe_ctx_destroy(madpipe_ctx *c) {
     if (!c) return;
     cudaSetDevice(c->device);
     cudaStreamSynchronize(c->stream);
+    c->profbuf.release();
     DevBuf *bufs[] = {&c->tables, &c->jobs, &c->tiles, &c->chains, &c->chain_data, &c->jl,
                       &c->counts, &c->roots, &c->trace, &c->stages, &c->scratch, &c->codes, &c->flags};
     for (DevBuf *b : bufs) b->release();
@@ -477,6 +482,10 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             persist_grid = std::min(n_tiles, ctx->num_sms * persist_blocks_per_sm(nmp, p_np, p_vb, nsg));
         }
         const bool per_launch = timed && ctx->per_launch_timing;
+        if (ctx->prof) {
+            CUDA_TRY(ctx, ctx->profbuf.ensure(8 * sizeof(unsigned long long)));
+            CUDA_TRY(ctx, cudaMemsetAsync(ctx->profbuf.p, 0, 8 * sizeof(unsigned long long), ctx->stream));
+        }
         if (per_launch && ctx->ev_pool.size() < (size_t)(2 * maxL)) {
             while (ctx->ev_pool.size() < (size_t)(2 * maxL)) {
                 cudaEvent_t ev;
@@ -492,7 +501,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             }
             if (ctx->kernel == 2)
                 launch_step_persist(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, p_np, p_vb, nsg,
-                                    persist_grid, ctx->stream);
+                                    persist_grid, (unsigned long long *)(ctx->prof ? ctx->profbuf.p : nullptr),
+                                    ctx->stream);
             else if (ctx->kernel == 1)
                 launch_step_tma(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, smem_tma, ctx->stream);
             else
@@ -505,6 +515,17 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         ctx->launches += 2;
         CUDA_TRY(ctx, cudaGetLastError());
         if (timed) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_b, ctx->stream));
+        if (ctx->prof && timed) {
+            unsigned long long pc[8];
+            CUDA_TRY(ctx, cudaMemcpy(pc, ctx->profbuf.p, sizeof pc, cudaMemcpyDeviceToHost));
+            fprintf(stderr,
+                    "[madpipe prof] batch of %d jobs, %d CTAs: producer total %.3g cyc/CTA: setup %.1f%% "
+                    "lists %.1f%% issue %.1f%% (empty waits %.1f%%); consumer warp0 waits on full %.1f%%; "
+                    "tiles %llu\n",
+                    nj, persist_grid, (double)pc[0] / std::max(1, persist_grid), 100.0 * pc[1] / std::max(1ull, pc[0]),
+                    100.0 * pc[2] / std::max(1ull, pc[0]), 100.0 * pc[3] / std::max(1ull, pc[0]),
+                    100.0 * pc[4] / std::max(1ull, pc[0]), 100.0 * pc[6] / std::max(1ull, pc[5]), pc[7]);
+        }
         if (hook) {
             int rc = hook->after_batch(ctx, ids, djobs);
             if (rc) return rc;

@@ -93,7 +93,10 @@ template <int NMP>
 __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job *__restrict__ jobs,
                                                                       const int32_t *__restrict__ tile_job,
                                                                       int n_tiles, int l, int np_max, int vb,
-                                                                      int nsg) {
+                                                                      int nsg, unsigned long long *prof) {
+    // prof (optional, MADPIPE_PROF=1): cycle counters [0] producer total, [1] tile setup,
+    // [2] list building, [3] issue, [4] producer waits on empty, [5] consumer total,
+    // [6] consumer waits on full, [7] tiles
     constexpr int C = NMP / 2;                       // 16-byte chunks per processor row
     constexpr bool ROW = NMP <= 16;
     constexpr int PER_ROW = ROW ? 1 : C;             // consumer threads per processor row
@@ -130,7 +133,10 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
         const int lpr = 32 / vb;                     // lanes per ring in the issue phase
         const int m_round = min(nsg, lpr);           // stages per ring per issue round
         const int iw = lane / lpr, ij = lane - (lane / lpr) * lpr;
+        long long t_p0 = clock64(), t_setup = 0, t_lists = 0, t_issue = 0, t_wempty = 0, n_tl = 0;
         for (int tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+            long long ta = clock64();
+            n_tl++;
             const int jid = tile_job[tile];
             __syncwarp();
             {   // cooperative copy of the job descriptor (one 8-byte word per lane)
@@ -168,6 +174,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             }
             if (np <= 0) continue;
             const int kmin = *J.kmin_l;
+            if (prof) { __syncwarp(); const long long tb = clock64(); t_setup += tb - ta; ta = tb; }
             const int per = 32 / vcount;              // k per pass (vcount <= 8)
             const int kk = lane / vcount, v2 = lane - kk * vcount;
             unsigned rowmask = 0;                     // lanes holding my row v2
@@ -196,6 +203,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                     cnt += __popc(mine);
                 }
                 __syncwarp();
+                if (prof) { const long long tb = clock64(); t_lists += tb - ta; ta = tb; }
                 // ---- issue: lane (iw, ij) takes stages ij, ij+m, ... of ring iw
                 const int n_w = __shfl_sync(0xffffffffu, cnt, iw < vcount ? iw : 0);
                 const bool my_ring = iw < vcount;
@@ -208,7 +216,11 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                         int s = p_sl[iw] + ij, use = p_us[iw];
                         if (s >= nsg) { s -= nsg; use++; }
                         const int slot = iw * nsg + s;
-                        if (use > 0) mbar_wait(empty0 + 8 * slot, (uint32_t)((use - 1) & 1));
+                        if (use > 0) {
+                            const long long tw = prof ? clock64() : 0;
+                            mbar_wait(empty0 + 8 * slot, (uint32_t)((use - 1) & 1));
+                            if (prof && lane == 0) t_wempty += clock64() - tw;
+                        }
                         SlotMeta &M = meta[slot];
                         M.out = out + (size_t)(v0 + iw) * rowlen + (size_t)p_lo * NMP;
                         M.flag = J.rowflag + (size_t)l * J.n_v + v0 + iw;
@@ -242,10 +254,19 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
                     }
                     __syncwarp();
                 }
+                if (prof) { const long long tb = clock64(); t_issue += tb - ta; ta = tb; }
                 if (done) break;
             }
         }
         __syncwarp();
+        if (prof && lane == 0) {
+            atomicAdd(prof + 0, (unsigned long long)(clock64() - t_p0));
+            atomicAdd(prof + 1, (unsigned long long)t_setup);
+            atomicAdd(prof + 2, (unsigned long long)t_lists);
+            atomicAdd(prof + 3, (unsigned long long)t_issue);
+            atomicAdd(prof + 4, (unsigned long long)t_wempty);
+            atomicAdd(prof + 7, (unsigned long long)n_tl);
+        }
         if (lane < vb) {   // terminate every ring
             const int w = lane;
             const int slot = w * nsg + p_sl[w];
@@ -275,12 +296,22 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
 #pragma unroll
     for (int i = 0; i < NB; i++) best[i] = MP_INF;
     int s = 0, phase = 0;
+    const long long t_c0 = clock64();
+    long long t_wfull = 0;
     for (;;) {
         const int slot = grp * nsg + s;
+        const long long tw = prof ? clock64() : 0;
         mbar_wait(full0 + 8 * slot, (uint32_t)phase);
+        if (prof) t_wfull += clock64() - tw;
         const SlotMeta &M = meta[slot];
         const int flags = M.flags;
-        if (flags & 4) break;
+        if (flags & 4) {
+            if (prof && lane == 0 && warp == 0) {
+                atomicAdd(prof + 5, (unsigned long long)(clock64() - t_c0));
+                atomicAdd(prof + 6, (unsigned long long)t_wfull);
+            }
+            break;
+        }
         const int np = M.np, n_m = M.n_m;
         const bool active = pp_off < np;
         if (!(flags & 2) && active) {
@@ -403,13 +434,13 @@ int persist_nsg(int np, int vb, int nmp) {
 }
 
 void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np,
-                         int vb, int nsg, int grid, cudaStream_t s) {
+                         int vb, int nsg, int grid, unsigned long long *prof, cudaStream_t s) {
     const int smem = vb * nsg * (np + 1) * nmp * 8;
     switch (nmp) {
 #define MP_CASE(N)                                                                                      \
     case N:                                                                                             \
         cudaFuncSetAttribute(step_persist_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
-        step_persist_kernel<N><<<grid, kPCons + 32, smem, s>>>(jobs, tile_job, n_tiles, l, np, vb, nsg); \
+        step_persist_kernel<N><<<grid, kPCons + 32, smem, s>>>(jobs, tile_job, n_tiles, l, np, vb, nsg, prof); \
         break;
         MP_CASE(2) MP_CASE(4) MP_CASE(8) MP_CASE(16) MP_CASE(32) MP_CASE(64)
 #undef MP_CASE
