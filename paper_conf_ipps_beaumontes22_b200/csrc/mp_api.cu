@@ -43,7 +43,8 @@ struct madpipe_ctx {
     bool own_stream = false;
     int64_t mem_budget = 0;
     std::string err;
-    DevBuf tables, jobs, tiles, chains, chain_data, jl, counts, roots, trace, stages, scratch, codes, flags;
+    DevBuf tables, jobs, tiles, chains, chain_data, jl, counts, roots, trace, stages, scratch, codes, flags,
+        tlist;
     cudaEvent_t ev_a = nullptr, ev_b = nullptr;
     double sweep_ms = 0.0, step_ms = 0.0;
     int64_t launches = 0;
@@ -236,7 +237,7 @@ extern "C" void madpipe_ctx_destroy(madpipe_ctx *c) {
     cudaStreamSynchronize(c->stream);
     c->profbuf.release();
     DevBuf *bufs[] = {&c->tables, &c->jobs, &c->tiles, &c->chains, &c->chain_data, &c->jl,
-                      &c->counts, &c->roots, &c->trace, &c->stages, &c->scratch, &c->codes, &c->flags};
+                      &c->counts, &c->roots, &c->trace, &c->stages, &c->scratch, &c->codes, &c->flags, &c->tlist};
     for (DevBuf *b : bufs) b->release();
     for (cudaEvent_t ev : c->ev_pool) cudaEventDestroy(ev);
     if (c->ev_a) cudaEventDestroy(c->ev_a);
@@ -446,15 +447,22 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         }
         int n_v_max = 0;
         if (ctx->kernel == 2) {
-            // transition codes of one layer: [job][v][maxL]
-            size_t total = 0;
-            for (auto &J : hjobs) { total += (size_t)J.n_v * (size_t)maxL; n_v_max = std::max(n_v_max, J.n_v); }
-            CUDA_TRY(ctx, ctx->codes.ensure(total * sizeof(int32_t)));
-            size_t off = 0, ftotal = 0;
+            // useful-transition lists of one layer: [job][v][maxL] entries + [job][v] counts
+            size_t total = 0, vtotal = 0;
             for (auto &J : hjobs) {
-                J.codes = (int32_t *)ctx->codes.p + off;
+                total += (size_t)J.n_v * (size_t)maxL;
+                vtotal += (size_t)J.n_v;
+                n_v_max = std::max(n_v_max, J.n_v);
+            }
+            CUDA_TRY(ctx, ctx->tlist.ensure(total * sizeof(TransEntry)));
+            CUDA_TRY(ctx, ctx->codes.ensure(vtotal * sizeof(int32_t)));
+            size_t off = 0, voff = 0, ftotal = 0;
+            for (auto &J : hjobs) {
+                J.tlist = (TransEntry *)ctx->tlist.p + off;
+                J.tcount = (int32_t *)ctx->codes.p + voff;
                 J.code_cap = maxL;
                 off += (size_t)J.n_v * (size_t)maxL;
+                voff += (size_t)J.n_v;
                 ftotal += (size_t)(J.L + 1) * (size_t)J.n_v;
             }
             CUDA_TRY(ctx, ctx->flags.ensure(ftotal * sizeof(uint32_t)));
@@ -496,7 +504,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         for (int l = 1; l <= maxL; l++) {
             if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1)], ctx->stream);
             if (ctx->kernel == 2) {
-                launch_trans(djobs, nj, n_v_max, l, ctx->stream);
+                launch_trans(djobs, nj, n_v_max, l, nmp, ctx->stream);
                 ctx->launches++;
             }
             if (ctx->kernel == 2)

@@ -48,6 +48,16 @@ struct Job {
     int32_t pad_;
     uint32_t *rowflag;  // [(L+1)][n_v]: 1 if row (l, v) holds a finite value (persist path)
     unsigned long long *useful;  // live relaxations whose source row is not all +inf
+    struct TransEntry *tlist;    // [n_v][code_cap] useful transitions of layer l (persist path)
+    int32_t *tcount;             // [n_v] their number
+    int32_t pad2_[2];
+};
+
+// One useful transition of layer l for delay row v, in ascending k (trans_kernel).
+struct TransEntry {
+    double U;        // U(k,l)
+    int32_t code;    // pack_trans(v', d, nf)
+    int32_t k;
 };
 
 // Result of a traceback, written by traceback_kernel.
@@ -85,7 +95,7 @@ int persist_blocks_per_sm(int nmp, int np, int vb, int nsg);
 void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
 int persist_nsg(int np, int vb, int nmp);
 void tma_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
-void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, cudaStream_t s);
+void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, cudaStream_t s);
 void launch_root(const Job *jobs, int n_jobs, int nmp, int32_t *jl_per_chain, double *root_out,
                  double *tau_out, cudaStream_t s);
 void launch_count(const Job *jobs, int n_jobs, unsigned long long *counts, cudaStream_t s);

@@ -255,52 +255,76 @@ void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, i
 }
 
 // ---------------------------------------------------------------------------
-// a3 for the persistent step kernel: every live/dead transition code of layer l,
-// computed by all SMs in parallel (one CTA per job x 8 delay rows) instead of
-// inside the step kernel's producer warp.  codes[v][kk] holds the transition of
-// k = kmin_l + kk; kmin_l = max(kmin_tau, kmin_W).  Also counts
-// the job's effective relaxations.
+// a3 (+ a4) for the persistent step kernel, computed by all SMs in parallel
+// (one warp per (job, delay row v)) instead of inside the step kernel's producer:
+// the base row A[l][v][0][*], and the list of USEFUL transitions of row
+// v in ascending k over the window [max(kmin_tau, kmin_W), l]:
+// live and with a source row A[k-1][v'] that holds a finite value
+// (a row that is +inf everywhere can only contribute +inf).  Also counts the
+// job's effective and useful relaxations.
 // ---------------------------------------------------------------------------
-__global__ void trans_kernel(const Job *jobs, int l) {
+__global__ void __launch_bounds__(256) trans_kernel(const Job *jobs, int l, int nmp) {
+    // one warp per delay row v of the job (8 rows per CTA)
     const Job &J = jobs[blockIdx.y];
     if (l > J.L) return;
-    const int v0 = blockIdx.x * 8;
-    if (v0 >= J.n_v) return;
-    const int vc = min(8, J.n_v - v0);
-    // the step kernel of layer l sets the row flags of slab l; clear them first
-    if (J.rowflag && threadIdx.x < vc) J.rowflag[(size_t)l * J.n_v + v0 + threadIdx.x] = 0u;
-    const int kmin = max(kmin_of(J, l), kmin_mem(J, l));
-    const int wl = l + 1 - kmin;   // may be <= 0
-    if (blockIdx.x == 0 && threadIdx.x == 0) *J.kmin_l = kmin;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int v = blockIdx.x * 8 + warp;
+    if (v >= J.n_v) return;
+    const size_t rowlen = (size_t)J.P * nmp;
     const double Ul = J.Up[l];
-    unsigned live = 0, useful = 0;
-    for (int e = threadIdx.x; e < vc * max(wl, 0); e += blockDim.x) {
-        const int vv = e / wl, kk = e - vv * wl;
-        const int k = kmin + kk;
-        int32_t tr = transition(J, k, l, v0 + vv, __dsub_rn(Ul, J.Up[k - 1]), nullptr);
-        if (tr >= 0) {
-            live++;
-            // a source row that is +inf everywhere can only contribute +inf (exact skip)
-            if (J.rowflag && J.rowflag[(size_t)(k - 1) * J.n_v + (tr & 0xFFFF)] == 0u)
-                tr = (int32_t)0x80000001;
-            else
-                useful++;
-        }
-        J.codes[(size_t)(v0 + vv) * J.code_cap + kk] = tr;
+    // base row p = 0 (reading Q10), and the row flag of (l, v): it is reset
+    // here and OR-ed by the step kernel for p >= 1
+    {
+        const double U1l = __dsub_rn(Ul, J.Up[0]);
+        int64_t d;
+        (void)transition(J, 1, l, v, U1l, &d);
+        const bool ok = U1l <= J.tau && d <= (int64_t)(J.n_m - 1);
+        double *o = J.table + (size_t)l * J.n_v * rowlen + (size_t)v * rowlen;
+        for (int m = lane; m < nmp; m += 32)
+            o[m] = (m < J.n_m && U1l <= J.tau && (int64_t)m + d <= (int64_t)(J.n_m - 1)) ? U1l : MP_INF;
+        if (lane == 0) J.rowflag[(size_t)l * J.n_v + v] = ok ? 1u : 0u;
     }
+    const int kmin = max(kmin_of(J, l), kmin_mem(J, l));
+    unsigned live = 0, useful = 0;
+    int n = 0;
+    TransEntry *list = J.tlist + (size_t)v * J.code_cap;
+    for (int kb = kmin; kb <= l; kb += 32) {
+        const int k = kb + lane;
+        int32_t tr = -1;
+        double Ukl = 0.0;
+        bool use = false;
+        if (k <= l) {
+            Ukl = __dsub_rn(Ul, J.Up[k - 1]);
+            tr = transition(J, k, l, v, Ukl, nullptr);
+            if (tr >= 0) {
+                live++;
+                // a source row that is +inf everywhere can only contribute +inf (exact skip)
+                use = J.rowflag[(size_t)(k - 1) * J.n_v + (tr & 0xFFFF)] != 0u;
+                useful += use;
+            }
+        }
+        const unsigned bal = __ballot_sync(0xffffffffu, use);
+        if (use) {
+            TransEntry e;
+            e.U = Ukl; e.code = tr; e.k = k;
+            list[n + __popc(bal & ((1u << lane) - 1u))] = e;
+        }
+        n += __popc(bal);
+    }
+    if (lane == 0) J.tcount[v] = n;
     for (int o = 16; o > 0; o >>= 1) {
         live += __shfl_xor_sync(0xffffffffu, live, o);
         useful += __shfl_xor_sync(0xffffffffu, useful, o);
     }
-    if ((threadIdx.x & 31) == 0 && live && J.P > 1) {
+    if (lane == 0 && live && J.P > 1) {
         const unsigned long long per = (unsigned long long)(J.P - 1) * (unsigned long long)J.n_m;
         atomicAdd(J.eff, (unsigned long long)live * per);
-        if (useful && J.useful) atomicAdd(J.useful, (unsigned long long)useful * per);
+        if (useful) atomicAdd(J.useful, (unsigned long long)useful * per);
     }
 }
 
-void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, cudaStream_t s) {
-    trans_kernel<<<dim3((n_v_max + 7) / 8, n_jobs), 256, 0, s>>>(jobs, l);
+void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, cudaStream_t s) {
+    trans_kernel<<<dim3((n_v_max + 7) / 8, n_jobs), 256, 0, s>>>(jobs, l, nmp);
 }
 
 // ---------------------------------------------------------------------------

@@ -5,24 +5,24 @@
 //   A[l][v][p][m] = clamp_tau( min over live k of
 //        N: A[k-1][v'][p-1][m]            (normal GPU fits)
 //        S: U(k,l) + A[k-1][v'][p][m+d]   (special GPU) ).
-// The transitions (k, v) -> (v', nf, d) of layer l were computed beforehand by
-// trans_kernel (a3) into J.codes for the window starting at *J.kmin_l; a
-// transition whose source row is +inf everywhere is already marked dead there.
+// The useful transitions (k, v) -> (v', nf, d) of layer l and the base row p = 0
+// were computed beforehand by trans_kernel (a3, a4) into J.tlist / J.tcount.
 //
 // Structure:
-//   * grid = resident CTAs (2 per SM); CTA c takes tiles c, c+G, c+2G, ...  A
-//     tile is vb delay rows x np processor rows of one job; every job of a launch
+//   * grid = resident CTAs (2 per SM); each CTA takes a contiguous range of
+//     tiles.  A tile is vb delay rows x np processor rows of one job; every job of a launch
 //     has the same P, hence the same tile geometry (passed as arguments).
 //   * per-row sub-rings: delay row w of a tile owns a ring of nsg one-row slots in
 //     shared memory, with its own full/empty mbarriers, consumed by its own warp
 //     group.  Every slot carries exactly one useful source row segment, so the
 //     bytes in flight per SM stay at the ring capacity whatever the liveness.
-//   * warp 8 is the producer.  Per tile it writes the base row p = 0 (a4),
-//     reads the window's codes 32 at a time (one coalesced load per lane), builds
-//     per-row lists of live k with ballots, and then issues, lane-parallel across
-//     rows and stages, one cp.async.bulk per live (k, row): the segment
-//     A[k-1][v'][p_lo-1 .. p_lo+np-1][*] into the row's next slot, completing on
-//     the slot's mbarrier.
+//   * warp 8 is the producer.  Per tile it reads, for each delay row, the list
+//     of useful transitions prepared by trans_kernel (U(k,l), code, k in
+//     ascending k) and issues, lane-parallel across rows and stages, one
+//     cp.async.bulk per entry: the segment A[k-1][v'][p_lo-1 .. p_lo+np-1][*]
+//     into the row's next slot, completing on the slot's mbarrier.  A CTA walks
+//     a contiguous range of tiles, so the job descriptor is reloaded only when
+//     the job changes.
 //   * warps 0-7 are consumers, one group per delay row.  ROW mode (NMP <= 16):
 //     a thread owns one (v, p) row of NMP levels as NMP/2 16-byte chunks held in
 //     a lane-rotated order (every quarter-warp's 16-byte shared loads hit 8
@@ -76,7 +76,6 @@ __device__ __forceinline__ double dmin(double a, double b) { return b < a ? b : 
 constexpr int kSlotsMax = 64;        // one-row slots per CTA (all rings)
 constexpr int kPCons = 256;          // consumer threads (8 warps); + 1 producer warp
 constexpr int kMaxVb = 8;            // delay rows (= rings) per tile
-constexpr int kSpan = 128;           // k per producer chunk
 
 struct SlotMeta {
     double *out;        // output row segment: A[l][v][p_lo][0]
@@ -105,9 +104,6 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
     __shared__ __align__(8) uint64_t empty[kSlotsMax];
     __shared__ SlotMeta meta[kSlotsMax];
     __shared__ Job pJ;                               // producer's copy of the current tile's job
-    __shared__ int16_t p_k[kMaxVb][kSpan];           // live k (offset in the chunk) per row
-    __shared__ int32_t p_code[kMaxVb][kSpan];        // its transition code
-    __shared__ double p_Uk[kSpan];                   // U(k,l) per k of the chunk
     __shared__ int p_sl[kMaxVb], p_us[kMaxVb];       // per ring: next slot, its use count
 
     const int tid = threadIdx.x;
@@ -134,18 +130,23 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
         const int m_round = min(nsg, lpr);           // stages per ring per issue round
         const int iw = lane / lpr, ij = lane - (lane / lpr) * lpr;
         long long t_p0 = clock64(), t_setup = 0, t_lists = 0, t_issue = 0, t_wempty = 0, n_tl = 0;
-        for (int tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        // contiguous tile range per CTA: consecutive tiles mostly share the job
+        const int t_begin = (int)((long long)n_tiles * blockIdx.x / gridDim.x);
+        const int t_end = (int)((long long)n_tiles * (blockIdx.x + 1) / gridDim.x);
+        int cur_jid = -1;
+        for (int tile = t_begin; tile < t_end; tile++) {
             long long ta = clock64();
             n_tl++;
             const int jid = tile_job[tile];
-            __syncwarp();
-            {   // cooperative copy of the job descriptor (one 8-byte word per lane)
+            if (jid != cur_jid) {   // cooperative copy of the job descriptor (one 8-byte word per lane)
                 static_assert(sizeof(Job) % 8 == 0 && sizeof(Job) <= 32 * 8 * 2, "Job size");
+                __syncwarp();
                 const uint64_t *src = reinterpret_cast<const uint64_t *>(jobs + jid);
                 uint64_t *dst = reinterpret_cast<uint64_t *>(&pJ);
                 for (int w = lane; w < (int)(sizeof(Job) / 8); w += 32) dst[w] = __ldg(src + w);
+                __syncwarp();
+                cur_jid = jid;
             }
-            __syncwarp();
             const Job &J = pJ;
             if (l > J.L) continue;
             const int t = tile - J.tile0;
@@ -154,109 +155,64 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             const int vcount = min(J.vb, J.n_v - v0);
             const int p_lo = 1 + pt * J.np;
             const int np = max(0, min(J.np, J.P - p_lo));
+            if (np <= 0) continue;
             const size_t rowlen = (size_t)J.P * NMP;
             const size_t slab = (size_t)J.n_v * rowlen;
             const uint32_t seg_bytes = (uint32_t)(np + 1) * NMP * 8u;
             double *out = J.table + (size_t)l * slab;
-            const double Ul = J.Up[l];
-            const double tau = J.tau;
-            const int n_m = J.n_m;
-            if (pt == 0 && lane < vcount) {          // base row p = 0 (Q10)
-                const int v = v0 + lane;
-                const double U1l = __dsub_rn(Ul, J.Up[0]);
-                int64_t d;
-                (void)transition(J, 1, l, v, U1l, &d);
-                double *o = out + (size_t)v * rowlen;
-#pragma unroll
-                for (int m = 0; m < NMP; m++)
-                    o[m] = (m < n_m && U1l <= tau && (int64_t)m + d <= (int64_t)(n_m - 1)) ? U1l : MP_INF;
-                if (U1l <= tau && d <= (int64_t)(n_m - 1)) atomicOr(J.rowflag + (size_t)l * J.n_v + v, 1u);
-            }
-            if (np <= 0) continue;
-            const int kmin = *J.kmin_l;
-            if (prof) { __syncwarp(); const long long tb = clock64(); t_setup += tb - ta; ta = tb; }
-            const int per = 32 / vcount;              // k per pass (vcount <= 8)
-            const int kk = lane / vcount, v2 = lane - kk * vcount;
-            unsigned rowmask = 0;                     // lanes holding my row v2
-            for (int q = 0; q < per; q++) rowmask |= 1u << (q * vcount + v2);
-            const int32_t *codes = J.codes + (size_t)(v0 + v2) * J.code_cap;
-            // (kmin may be l+1: an empty window still runs one chunk, whose rows all get a
-            // closing stage, so every consumer group sees the end of every tile)
-            for (int kc0 = kmin;; kc0 += kSpan) {
-                const int kc1 = min(l + 1, kc0 + kSpan);
-                const bool done = kc1 > l;
-                // ---- per-row lists of live k in [kc0, kc1)
-                int cnt = 0;                          // live entries of row v2 so far (per lane)
-                for (int kb = kc0; kb < kc1; kb += per) {
-                    const int k = kb + kk;
-                    const bool valid = kk < per && k < kc1;
-                    const int32_t tr = valid ? __ldg(codes + (k - kmin)) : -1;
-                    if (valid && v2 == 0) p_Uk[k - kc0] = __dsub_rn(Ul, __ldg(J.Up + k - 1));
-                    const unsigned live = __ballot_sync(0xffffffffu, tr >= 0) & (valid ? 0xffffffffu : 0u);
-                    const unsigned mine = __ballot_sync(0xffffffffu, tr >= 0) & rowmask;
-                    if (tr >= 0) {
-                        const int pos = cnt + __popc(mine & ((1u << lane) - 1u));
-                        p_k[v2][pos] = (int16_t)(k - kc0);
-                        p_code[v2][pos] = tr;
+            const bool my_ring = iw < vcount;
+            // number of useful transitions of my ring's row (trans_kernel)
+            const int n_w = my_ring ? __ldg(J.tcount + v0 + iw) : 0;
+            const TransEntry *list = J.tlist + (size_t)(v0 + (my_ring ? iw : 0)) * J.code_cap;
+            const int n_eff = my_ring ? (n_w > 0 ? n_w : 1) : 0;   // 1 = closing stage without data
+            int max_n = n_eff;
+            for (int o = 16; o > 0; o >>= 1) max_n = max(max_n, __shfl_xor_sync(0xffffffffu, max_n, o));
+            if (prof) { const long long tb = clock64(); t_setup += tb - ta; ta = tb; }
+            // ---- issue: lane (iw, ij) takes stages ij, ij+m, ... of ring iw
+            for (int r0 = 0; r0 < max_n; r0 += m_round) {
+                const int q = r0 + ij;
+                if (my_ring && ij < m_round && q < n_eff) {
+                    TransEntry e;
+                    if (n_w > 0) e = list[q];
+                    int s = p_sl[iw] + ij, use = p_us[iw];
+                    if (s >= nsg) { s -= nsg; use++; }
+                    const int slot = iw * nsg + s;
+                    if (use > 0) {
+                        const long long tw = prof ? clock64() : 0;
+                        mbar_wait(empty0 + 8 * slot, (uint32_t)((use - 1) & 1));
+                        if (prof && lane == 0) t_wempty += clock64() - tw;
                     }
-                    (void)live;
-                    cnt += __popc(mine);
+                    SlotMeta &M = meta[slot];
+                    M.out = out + (size_t)(v0 + iw) * rowlen + (size_t)p_lo * NMP;
+                    M.flag = J.rowflag + (size_t)l * J.n_v + v0 + iw;
+                    M.tau = J.tau;
+                    M.np = np;
+                    M.n_m = (int16_t)J.n_m;
+                    if (n_w == 0) {
+                        M.flags = 1 | 2;
+                        M.tr = -1;
+                        mbar_arrive(full0 + 8 * slot);
+                    } else {
+                        bulk_g2s(ring_s + 8u * (uint32_t)(slot * seg_doubles),
+                                 J.table + (size_t)(e.k - 1) * slab + (size_t)(e.code & 0xFFFF) * rowlen +
+                                     (size_t)(p_lo - 1) * NMP,
+                                 seg_bytes, full0 + 8 * slot);
+                        M.flags = (int16_t)(q == n_w - 1 ? 1 : 0);
+                        M.tr = e.code;
+                        M.U = e.U;
+                        mbar_arrive_expect_tx(full0 + 8 * slot, seg_bytes);
+                    }
                 }
                 __syncwarp();
-                if (prof) { const long long tb = clock64(); t_lists += tb - ta; ta = tb; }
-                // ---- issue: lane (iw, ij) takes stages ij, ij+m, ... of ring iw
-                const int n_w = __shfl_sync(0xffffffffu, cnt, iw < vcount ? iw : 0);
-                const bool my_ring = iw < vcount;
-                const int n_eff = my_ring ? (n_w > 0 ? n_w : (done ? 1 : 0)) : 0;   // 1 = closing stage
-                int max_n = n_eff;
-                for (int o = 16; o > 0; o >>= 1) max_n = max(max_n, __shfl_xor_sync(0xffffffffu, max_n, o));
-                for (int r0 = 0; r0 < max_n; r0 += m_round) {
-                    const int q = r0 + ij;
-                    if (my_ring && ij < m_round && q < n_eff) {
-                        int s = p_sl[iw] + ij, use = p_us[iw];
-                        if (s >= nsg) { s -= nsg; use++; }
-                        const int slot = iw * nsg + s;
-                        if (use > 0) {
-                            const long long tw = prof ? clock64() : 0;
-                            mbar_wait(empty0 + 8 * slot, (uint32_t)((use - 1) & 1));
-                            if (prof && lane == 0) t_wempty += clock64() - tw;
-                        }
-                        SlotMeta &M = meta[slot];
-                        M.out = out + (size_t)(v0 + iw) * rowlen + (size_t)p_lo * NMP;
-                        M.flag = J.rowflag + (size_t)l * J.n_v + v0 + iw;
-                        M.tau = tau;
-                        M.np = np;
-                        M.n_m = (int16_t)n_m;
-                        if (n_w == 0) {              // closing stage without data
-                            M.flags = 1 | 2;
-                            M.tr = -1;
-                            mbar_arrive(full0 + 8 * slot);
-                        } else {
-                            const int kofs = p_k[iw][q];
-                            const int32_t tr = p_code[iw][q];
-                            const int k = kc0 + kofs;
-                            bulk_g2s(ring_s + 8u * (uint32_t)(slot * seg_doubles),
-                                     J.table + (size_t)(k - 1) * slab + (size_t)(tr & 0xFFFF) * rowlen +
-                                         (size_t)(p_lo - 1) * NMP,
-                                     seg_bytes, full0 + 8 * slot);
-                            M.flags = (int16_t)(done && q == n_w - 1 ? 1 : 0);
-                            M.tr = tr;
-                            M.U = p_Uk[kofs];
-                            mbar_arrive_expect_tx(full0 + 8 * slot, seg_bytes);
-                        }
-                    }
-                    __syncwarp();
-                    if (my_ring && ij == 0) {         // advance ring iw by the stages of this round
-                        const int adv = max(0, min(m_round, n_eff - r0));
-                        int s = p_sl[iw] + adv;
-                        if (s >= nsg) { s -= nsg; p_us[iw]++; }
-                        p_sl[iw] = s;
-                    }
-                    __syncwarp();
+                if (my_ring && ij == 0) {         // advance ring iw by the stages of this round
+                    const int adv = max(0, min(m_round, n_eff - r0));
+                    int s = p_sl[iw] + adv;
+                    if (s >= nsg) { s -= nsg; p_us[iw]++; }
+                    p_sl[iw] = s;
                 }
-                if (prof) { const long long tb = clock64(); t_issue += tb - ta; ta = tb; }
-                if (done) break;
+                __syncwarp();
             }
+            if (prof) { const long long tb = clock64(); t_issue += tb - ta; ta = tb; }
         }
         __syncwarp();
         if (prof && lane == 0) {
