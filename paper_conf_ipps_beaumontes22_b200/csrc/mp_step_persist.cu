@@ -9,20 +9,19 @@
 // were computed beforehand by trans_kernel (a3, a4) into J.tlist / J.tcount.
 //
 // Structure:
-//   * grid = resident CTAs (2 per SM); each CTA takes a contiguous range of
-//     tiles.  A tile is vb delay rows x np processor rows of one job; every job of a launch
+//   * grid = resident CTAs (2 per SM).  A tile is vb delay rows x np processor rows of one job; every job of a launch
 //     has the same P, hence the same tile geometry (passed as arguments).
 //   * per-row sub-rings: delay row w of a tile owns a ring of nsg one-row slots in
 //     shared memory, with its own full/empty mbarriers, consumed by its own warp
 //     group.  Every slot carries exactly one useful source row segment, so the
 //     bytes in flight per SM stay at the ring capacity whatever the liveness.
-//   * warp 8 is the producer.  Per tile it reads, for each delay row, the list
+//   * warps 8-11 are producers; producer i feeds rings i, i+4.  Per tile it reads, for each owned delay row, the list
 //     of useful transitions prepared by trans_kernel (U(k,l), code, k in
 //     ascending k) and issues, lane-parallel across rows and stages, one
 //     cp.async.bulk per entry: the segment A[k-1][v'][p_lo-1 .. p_lo+np-1][*]
-//     into the row's next slot, completing on the slot's mbarrier.  A CTA walks
-//     a contiguous range of tiles, so the job descriptor is reloaded only when
-//     the job changes.
+//     into the row's next slot, completing on the slot's mbarrier.  Tiles are
+//     dealt to CTAs in interleaved blocks of 8 consecutive tiles (load balance;
+//     the job descriptor is reloaded only when the job changes).
 //   * warps 0-7 are consumers, one group per delay row.  ROW mode (NMP <= 16):
 //     a thread owns one (v, p) row of NMP levels as NMP/2 16-byte chunks held in
 //     a lane-rotated order (every quarter-warp's 16-byte shared loads hit 8
@@ -74,7 +73,9 @@ __device__ __forceinline__ double dmin(double a, double b) { return b < a ? b : 
 }  // namespace
 
 constexpr int kSlotsMax = 64;        // one-row slots per CTA (all rings)
-constexpr int kPCons = 256;          // consumer threads (8 warps); + 1 producer warp
+constexpr int kPCons = 256;          // consumer threads (8 warps)
+constexpr int kProd = 4;             // producer warps (ring w is fed by producer w % kProd)
+constexpr int kTileBlock = 8;        // tiles per interleaved block
 constexpr int kMaxVb = 8;            // delay rows (= rings) per tile
 
 struct SlotMeta {
@@ -89,7 +90,7 @@ struct SlotMeta {
 };
 
 template <int NMP>
-__global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job *__restrict__ jobs,
+__global__ void __launch_bounds__(kPCons + 32 * kProd, 2) step_persist_kernel(const Job *__restrict__ jobs,
                                                                       const int32_t *__restrict__ tile_job,
                                                                       int n_tiles, int l, int np_max, int vb,
                                                                       int nsg, unsigned long long *prof) {
@@ -103,7 +104,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
     __shared__ __align__(8) uint64_t full[kSlotsMax];
     __shared__ __align__(8) uint64_t empty[kSlotsMax];
     __shared__ SlotMeta meta[kSlotsMax];
-    __shared__ Job pJ;                               // producer's copy of the current tile's job
+    __shared__ Job pJs[kProd];                       // each producer's copy of its tile's job
     __shared__ int p_sl[kMaxVb], p_us[kMaxVb];       // per ring: next slot, its use count
 
     const int tid = threadIdx.x;
@@ -124,17 +125,22 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
     __syncthreads();
     const double *ring = reinterpret_cast<const double *>(dsm);
 
-    if (warp == kPCons / 32) {
-        // ======================================================= producer warp
-        const int lpr = 32 / vb;                     // lanes per ring in the issue phase
+    if (warp >= kPCons / 32) {
+        // ======================================================= producer warps
+        const int pw = warp - kPCons / 32;           // producer index: rings pw, pw+kProd, ...
+        Job &pJ = pJs[pw];
+        const int my_rings = vb > pw ? (vb - pw + kProd - 1) / kProd : 0;
+        const int lpr = my_rings > 0 ? 32 / my_rings : 32;   // lanes per owned ring
         const int m_round = min(nsg, lpr);           // stages per ring per issue round
-        const int iw = lane / lpr, ij = lane - (lane / lpr) * lpr;
+        const int ir = lane / lpr, ij = lane - (lane / lpr) * lpr;
+        const int iw = pw + ir * kProd;              // the ring this lane serves
         long long t_p0 = clock64(), t_setup = 0, t_lists = 0, t_issue = 0, t_wempty = 0, n_tl = 0;
-        // contiguous tile range per CTA: consecutive tiles mostly share the job
-        const int t_begin = (int)((long long)n_tiles * blockIdx.x / gridDim.x);
-        const int t_end = (int)((long long)n_tiles * (blockIdx.x + 1) / gridDim.x);
         int cur_jid = -1;
-        for (int tile = t_begin; tile < t_end; tile++) {
+        // blocks of kTileBlock consecutive tiles, interleaved over the CTAs (balance +
+        // job-descriptor reuse)
+        for (int b0 = blockIdx.x * kTileBlock; b0 < n_tiles; b0 += gridDim.x * kTileBlock)
+        for (int tile = b0; tile < min(n_tiles, b0 + kTileBlock); tile++) {
+            if (my_rings == 0) break;
             long long ta = clock64();
             n_tl++;
             const int jid = tile_job[tile];
@@ -160,7 +166,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             const size_t slab = (size_t)J.n_v * rowlen;
             const uint32_t seg_bytes = (uint32_t)(np + 1) * NMP * 8u;
             double *out = J.table + (size_t)l * slab;
-            const bool my_ring = iw < vcount;
+            const bool my_ring = ir < my_rings && iw < vcount;
             // number of useful transitions of my ring's row (trans_kernel)
             const int n_w = my_ring ? __ldg(J.tcount + v0 + iw) : 0;
             const TransEntry *list = J.tlist + (size_t)(v0 + (my_ring ? iw : 0)) * J.code_cap;
@@ -215,7 +221,7 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             if (prof) { const long long tb = clock64(); t_issue += tb - ta; ta = tb; }
         }
         __syncwarp();
-        if (prof && lane == 0) {
+        if (prof && lane == 0 && pw == 0) {
             atomicAdd(prof + 0, (unsigned long long)(clock64() - t_p0));
             atomicAdd(prof + 1, (unsigned long long)t_setup);
             atomicAdd(prof + 2, (unsigned long long)t_lists);
@@ -223,8 +229,8 @@ __global__ void __launch_bounds__(kPCons + 32, 2) step_persist_kernel(const Job 
             atomicAdd(prof + 4, (unsigned long long)t_wempty);
             atomicAdd(prof + 7, (unsigned long long)n_tl);
         }
-        if (lane < vb) {   // terminate every ring
-            const int w = lane;
+        if (lane < my_rings) {   // terminate my rings
+            const int w = pw + lane * kProd;
             const int slot = w * nsg + p_sl[w];
             if (p_us[w] > 0) mbar_wait(empty0 + 8 * slot, (uint32_t)((p_us[w] - 1) & 1));
             meta[slot].flags = 4;
@@ -396,7 +402,7 @@ void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, 
 #define MP_CASE(N)                                                                                      \
     case N:                                                                                             \
         cudaFuncSetAttribute(step_persist_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
-        step_persist_kernel<N><<<grid, kPCons + 32, smem, s>>>(jobs, tile_job, n_tiles, l, np, vb, nsg, prof); \
+        step_persist_kernel<N><<<grid, kPCons + 32 * kProd, smem, s>>>(jobs, tile_job, n_tiles, l, np, vb, nsg, prof); \
         break;
         MP_CASE(2) MP_CASE(4) MP_CASE(8) MP_CASE(16) MP_CASE(32) MP_CASE(64)
 #undef MP_CASE
@@ -410,7 +416,7 @@ int persist_blocks_per_sm(int nmp, int np, int vb, int nsg) {
 #define MP_OCC(N)                                                                                       \
     case N:                                                                                             \
         cudaFuncSetAttribute(step_persist_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, step_persist_kernel<N>, kPCons + 32, smem);  \
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, step_persist_kernel<N>, kPCons + 32 * kProd, smem);  \
         break;
         MP_OCC(2) MP_OCC(4) MP_OCC(8) MP_OCC(16) MP_OCC(32) MP_OCC(64)
 #undef MP_OCC
