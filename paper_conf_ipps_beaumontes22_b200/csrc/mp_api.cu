@@ -53,6 +53,8 @@ struct madpipe_ctx {
     int per_launch_timing = 0;
     int kernel = 2;           // MADPIPE_KERNEL: v1 = plain loads, tma = per-tile TMA, persist (default)
     int prof = 0;             // MADPIPE_PROF=1: cycle counters of the persistent step kernel to stderr
+    int n_prod = 4;           // MADPIPE_NPROD: producer warps of the persistent step kernel (1..4)
+    int tile_block = 8;       // MADPIPE_TILE_BLOCK: consecutive tiles per interleaved block
     DevBuf profbuf;
     int num_sms = 148;
     std::vector<cudaEvent_t> ev_pool;
@@ -225,6 +227,8 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stre
     cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device);
     const char *pf = getenv("MADPIPE_PROF");
     c->prof = pf && pf[0] == '1';
+    if (const char *e = getenv("MADPIPE_NPROD")) c->n_prod = std::max(1, std::min(4, atoi(e)));
+    if (const char *e = getenv("MADPIPE_TILE_BLOCK")) c->tile_block = std::max(1, atoi(e));
     cudaEventCreate(&c->ev_a);
     cudaEventCreate(&c->ev_b);
     *out = c;
@@ -487,7 +491,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             p_vb = hjobs[0].vb;
             nsg = persist_nsg(p_np, p_vb, nmp);
             if (nsg < 2) return fail(ctx, MADPIPE_EINVAL, "row segment too large for the step kernel ring");
-            persist_grid = std::min(n_tiles, ctx->num_sms * persist_blocks_per_sm(nmp, p_np, p_vb, nsg));
+            persist_grid = std::min(n_tiles, ctx->num_sms * persist_blocks_per_sm(nmp, p_np, p_vb, nsg, ctx->n_prod));
         }
         const bool per_launch = timed && ctx->per_launch_timing;
         if (ctx->prof) {
@@ -510,7 +514,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             if (ctx->kernel == 2)
                 launch_step_persist(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, p_np, p_vb, nsg,
                                     persist_grid, (unsigned long long *)(ctx->prof ? ctx->profbuf.p : nullptr),
-                                    ctx->stream);
+                                    ctx->n_prod, ctx->tile_block, ctx->stream);
             else if (ctx->kernel == 1)
                 launch_step_tma(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, smem_tma, ctx->stream);
             else

@@ -90,8 +90,9 @@ void launch_step_tma(const Job *jobs, const int32_t *tile_job, int n_tiles, int 
                      cudaStream_t s);
 int tma_smem_bytes(int vb, int np, int nmp);
 void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np,
-                         int vb, int nsg, int grid, unsigned long long *prof, cudaStream_t s);
-int persist_blocks_per_sm(int nmp, int np, int vb, int nsg);
+                         int vb, int nsg, int grid, unsigned long long *prof, int n_prod, int tile_block,
+                         cudaStream_t s);
+int persist_blocks_per_sm(int nmp, int np, int vb, int nsg, int n_prod);
 void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
 int persist_nsg(int np, int vb, int nmp);
 void tma_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);

@@ -15,7 +15,7 @@
 //     shared memory, with its own full/empty mbarriers, consumed by its own warp
 //     group.  Every slot carries exactly one useful source row segment, so the
 //     bytes in flight per SM stay at the ring capacity whatever the liveness.
-//   * warps 8-11 are producers; producer i feeds rings i, i+4.  Per tile it reads, for each owned delay row, the list
+//   * warps 8.. are producers (n_prod, default 4); producer i feeds rings i, i+n_prod.  Per tile it reads, for each owned delay row, the list
 //     of useful transitions prepared by trans_kernel (U(k,l), code, k in
 //     ascending k) and issues, lane-parallel across rows and stages, one
 //     cp.async.bulk per entry: the segment A[k-1][v'][p_lo-1 .. p_lo+np-1][*]
@@ -74,8 +74,7 @@ __device__ __forceinline__ double dmin(double a, double b) { return b < a ? b : 
 
 constexpr int kSlotsMax = 64;        // one-row slots per CTA (all rings)
 constexpr int kPCons = 256;          // consumer threads (8 warps)
-constexpr int kProd = 4;             // producer warps (ring w is fed by producer w % kProd)
-constexpr int kTileBlock = 8;        // tiles per interleaved block
+constexpr int kProdMax = 4;          // producer warps (ring w is fed by producer w % n_prod)
 constexpr int kMaxVb = 8;            // delay rows (= rings) per tile
 
 struct SlotMeta {
@@ -90,10 +89,11 @@ struct SlotMeta {
 };
 
 template <int NMP>
-__global__ void __launch_bounds__(kPCons + 32 * kProd, 2) step_persist_kernel(const Job *__restrict__ jobs,
+__global__ void __launch_bounds__(kPCons + 32 * kProdMax, 2) step_persist_kernel(const Job *__restrict__ jobs,
                                                                       const int32_t *__restrict__ tile_job,
                                                                       int n_tiles, int l, int np_max, int vb,
-                                                                      int nsg, unsigned long long *prof) {
+                                                                      int nsg, unsigned long long *prof,
+                                                                      int n_prod, int tile_block) {
     // prof (optional, MADPIPE_PROF=1): cycle counters [0] producer total, [1] tile setup,
     // [2] list building, [3] issue, [4] producer waits on empty, [5] consumer total,
     // [6] consumer waits on full, [7] tiles
@@ -104,7 +104,7 @@ __global__ void __launch_bounds__(kPCons + 32 * kProd, 2) step_persist_kernel(co
     __shared__ __align__(8) uint64_t full[kSlotsMax];
     __shared__ __align__(8) uint64_t empty[kSlotsMax];
     __shared__ SlotMeta meta[kSlotsMax];
-    __shared__ Job pJs[kProd];                       // each producer's copy of its tile's job
+    __shared__ Job pJs[kProdMax];                    // each producer's copy of its tile's job
     __shared__ int p_sl[kMaxVb], p_us[kMaxVb];       // per ring: next slot, its use count
 
     const int tid = threadIdx.x;
@@ -129,17 +129,17 @@ __global__ void __launch_bounds__(kPCons + 32 * kProd, 2) step_persist_kernel(co
         // ======================================================= producer warps
         const int pw = warp - kPCons / 32;           // producer index: rings pw, pw+kProd, ...
         Job &pJ = pJs[pw];
-        const int my_rings = vb > pw ? (vb - pw + kProd - 1) / kProd : 0;
+        const int my_rings = vb > pw ? (vb - pw + n_prod - 1) / n_prod : 0;
         const int lpr = my_rings > 0 ? 32 / my_rings : 32;   // lanes per owned ring
         const int m_round = min(nsg, lpr);           // stages per ring per issue round
         const int ir = lane / lpr, ij = lane - (lane / lpr) * lpr;
-        const int iw = pw + ir * kProd;              // the ring this lane serves
+        const int iw = pw + ir * n_prod;             // the ring this lane serves
         long long t_p0 = clock64(), t_setup = 0, t_lists = 0, t_issue = 0, t_wempty = 0, n_tl = 0;
         int cur_jid = -1;
         // blocks of kTileBlock consecutive tiles, interleaved over the CTAs (balance +
         // job-descriptor reuse)
-        for (int b0 = blockIdx.x * kTileBlock; b0 < n_tiles; b0 += gridDim.x * kTileBlock)
-        for (int tile = b0; tile < min(n_tiles, b0 + kTileBlock); tile++) {
+        for (int b0 = blockIdx.x * tile_block; b0 < n_tiles; b0 += gridDim.x * tile_block)
+        for (int tile = b0; tile < min(n_tiles, b0 + tile_block); tile++) {
             if (my_rings == 0) break;
             long long ta = clock64();
             n_tl++;
@@ -230,7 +230,7 @@ __global__ void __launch_bounds__(kPCons + 32 * kProd, 2) step_persist_kernel(co
             atomicAdd(prof + 7, (unsigned long long)n_tl);
         }
         if (lane < my_rings) {   // terminate my rings
-            const int w = pw + lane * kProd;
+            const int w = pw + lane * n_prod;
             const int slot = w * nsg + p_sl[w];
             if (p_us[w] > 0) mbar_wait(empty0 + 8 * slot, (uint32_t)((p_us[w] - 1) & 1));
             meta[slot].flags = 4;
@@ -396,27 +396,28 @@ int persist_nsg(int np, int vb, int nmp) {
 }
 
 void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np,
-                         int vb, int nsg, int grid, unsigned long long *prof, cudaStream_t s) {
+                         int vb, int nsg, int grid, unsigned long long *prof, int n_prod, int tile_block,
+                         cudaStream_t s) {
     const int smem = vb * nsg * (np + 1) * nmp * 8;
     switch (nmp) {
 #define MP_CASE(N)                                                                                      \
     case N:                                                                                             \
         cudaFuncSetAttribute(step_persist_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
-        step_persist_kernel<N><<<grid, kPCons + 32 * kProd, smem, s>>>(jobs, tile_job, n_tiles, l, np, vb, nsg, prof); \
+        step_persist_kernel<N><<<grid, kPCons + 32 * n_prod, smem, s>>>(jobs, tile_job, n_tiles, l, np, vb, nsg, prof, n_prod, tile_block); \
         break;
         MP_CASE(2) MP_CASE(4) MP_CASE(8) MP_CASE(16) MP_CASE(32) MP_CASE(64)
 #undef MP_CASE
     }
 }
 
-int persist_blocks_per_sm(int nmp, int np, int vb, int nsg) {
+int persist_blocks_per_sm(int nmp, int np, int vb, int nsg, int n_prod) {
     const int smem = vb * nsg * (np + 1) * nmp * 8;
     int n = 0;
     switch (nmp) {
 #define MP_OCC(N)                                                                                       \
     case N:                                                                                             \
         cudaFuncSetAttribute(step_persist_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, step_persist_kernel<N>, kPCons + 32 * kProd, smem);  \
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, step_persist_kernel<N>, kPCons + 32 * n_prod, smem);  \
         break;
         MP_OCC(2) MP_OCC(4) MP_OCC(8) MP_OCC(16) MP_OCC(32) MP_OCC(64)
 #undef MP_OCC
