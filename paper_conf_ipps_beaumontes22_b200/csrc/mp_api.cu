@@ -54,7 +54,7 @@ struct madpipe_ctx {
     int kernel = 2;           // MADPIPE_KERNEL: v1 = plain loads, tma = per-tile TMA, persist (default)
     int prof = 0;             // MADPIPE_PROF=1: cycle counters of the persistent step kernel to stderr
     int n_prod = 4;           // MADPIPE_NPROD: producer warps of the persistent step kernel (1..4)
-    int tile_block = 8;       // MADPIPE_TILE_BLOCK: consecutive tiles per interleaved block
+    int tile_block = 1;       // MADPIPE_TILE_BLOCK: consecutive tiles per interleaved block (1 = round-robin)
     DevBuf profbuf;
     int num_sms = 148;
     std::vector<cudaEvent_t> ev_pool;

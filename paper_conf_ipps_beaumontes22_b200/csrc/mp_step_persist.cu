@@ -20,8 +20,8 @@
 //     ascending k) and issues, lane-parallel across rows and stages, one
 //     cp.async.bulk per entry: the segment A[k-1][v'][p_lo-1 .. p_lo+np-1][*]
 //     into the row's next slot, completing on the slot's mbarrier.  Tiles are
-//     dealt to CTAs in interleaved blocks of 8 consecutive tiles (load balance;
-//     the job descriptor is reloaded only when the job changes).
+//     dealt to CTAs round-robin (tile_block = 1, measured best: candidates differ
+//     in cost, interleaving balances them).
 //   * warps 0-7 are consumers, one group per delay row.  ROW mode (NMP <= 16):
 //     a thread owns one (v, p) row of NMP levels as NMP/2 16-byte chunks held in
 //     a lane-rotated order (every quarter-warp's 16-byte shared loads hit 8
