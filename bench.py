@@ -47,6 +47,8 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--force-dist", action="store_true",
+                    help="use the multi-GPU controller (sweep + NCCL all-reduce + resolve) even at N=1")
     return ap.parse_args()
 
 
@@ -177,7 +179,8 @@ def main():
     rank, world, local = env_rank()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if world > 1:
+    use_dist = world > 1 or args.force_dist
+    if use_dist:
         dist.init_process_group("nccl", device_id=dev)
     stream = torch.cuda.current_stream(dev)
     ctx = mp.Context(local, stream=stream.cuda_stream)
@@ -193,7 +196,7 @@ def main():
 
     def step(chain, early_exit=False):
         """One solve; returns (result, this rank's cell updates, launches, step-kernel ms)."""
-        if world == 1:
+        if not use_dist:
             if chain is dchain:
                 res = ctx.solve_dev(dchain, *a, early_exit=early_exit)
             else:
@@ -210,7 +213,7 @@ def main():
         for _ in range(k):
             flush.zero_()
             torch.cuda.synchronize(dev)
-            if world > 1:
+            if use_dist:
                 dist.barrier()
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
@@ -240,13 +243,13 @@ def main():
     ee_run = timed(dchain, args.steps, early_exit=True)
 
     def reduce(x, op):
-        if world == 1:
+        if not use_dist:
             return x
         t = torch.tensor([float(x)], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=op)
         return t.item()
 
-    SUM, MAX = (dist.ReduceOp.SUM, dist.ReduceOp.MAX) if world > 1 else (None, None)
+    SUM, MAX = (dist.ReduceOp.SUM, dist.ReduceOp.MAX) if use_dist else (None, None)
     K = args.steps
     tot_ms = reduce(sum(main_run["dev_ms"]), MAX)
     cu_step = reduce(main_run["cu"][-1], SUM)
@@ -267,7 +270,7 @@ def main():
                "ms_per_step": max(e2e_ms, 1e3 * e2e_wall) / K,
                "entry": "madpipe_solve (N=1) / madpipe_sweep+resolve (N>1) on pinned host arrays"}
     if rank != 0:
-        if world > 1:
+        if use_dist:
             dist.destroy_process_group()
         return
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) \
@@ -290,8 +293,9 @@ def main():
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K,
         "warmup": args.warmup, "ms_per_step": tot_ms / K, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic (chaingen, seeded)",
-        "config": {**workload(cfg), "parallelism": "candidates interleaved over %d rank(s), 1 NCCL "
-                                                   "all-reduce(MIN)" % world,
+        "config": {**workload(cfg), "parallelism": ("candidates interleaved over %d rank(s), 1 NCCL "
+                                                    "all-reduce(MIN) per solve" % world) if use_dist
+                   else "1 GPU, madpipe_solve_dev",
                    "l2": "DP tables >> L2 (%.0f MB per candidate) and a %d MB L2 flush between steps"
                          % ((cfg["L"] + 1) * cfg["P"] * cfg["n_delay"] * cfg["n_mem"] * 8 / 1e6,
                             L2_FLUSH_BYTES >> 20)},
@@ -312,7 +316,7 @@ def main():
         "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(), "cpu_baseline": cpu,
     }
     print(json.dumps(line), flush=True)
-    if world > 1:
+    if use_dist:
         dist.destroy_process_group()
 
 
