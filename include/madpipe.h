@@ -70,7 +70,11 @@ typedef struct {
     int32_t n_delay;    /* levels of the delay V, 2..65535                               */
     int32_t n_periods;  /* candidate periods, uniform on [lb, ub] (P:205 l.1-2, Q14), >= 1 */
     int32_t v_range;    /* madpipe_vrange                                                 */
-    int32_t early_exit; /* 0: evaluate every candidate; 1: stop at the first feasible one  */
+    int32_t early_exit; /* 0: evaluate every candidate; 1: ascending, stop at the first
+                           feasible one (exact); 2: coarse-to-fine (every ~sqrt(n_periods)-th
+                           candidate, then the gap below the first feasible one; equal to
+                           the full sweep when feasibility is monotone in the period, P:199;
+                           madpipe_solve / _solve_dev only -- elsewhere 2 acts as 1)        */
 } madpipe_disc;
 
 /* Result of a solve (the decisions along the optimal path give the

@@ -133,7 +133,8 @@ class HostChain:
 
 
 def make_disc(n_mem, n_delay, n_periods, v_range=VRANGE_PAPER, early_exit=False) -> Disc:
-    return Disc(int(n_mem), int(n_delay), int(n_periods), int(v_range), 1 if early_exit else 0)
+    ee = int(early_exit) if not isinstance(early_exit, bool) else (1 if early_exit else 0)
+    return Disc(int(n_mem), int(n_delay), int(n_periods), int(v_range), ee)
 
 
 class AllocBuf:

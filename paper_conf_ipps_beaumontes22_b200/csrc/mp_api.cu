@@ -702,16 +702,55 @@ int solve_common(madpipe_ctx *ctx, const madpipe_chain *chain, bool on_device, i
     rc = upload_chains(ctx, cs, cd);
     if (rc) return rc;
     CUDA_TRY(ctx, ctx->jl.ensure(sizeof(int32_t)));
-    { int _r = fill_int_max(ctx, (int32_t *)ctx->jl.p, 1); if (_r) return _r; }
-    std::vector<uint64_t> counts;
-    rc = run_jobs(ctx, cs, cd, disc, shard_jobs(0, disc->n_periods, 0, 1), (int32_t *)ctx->jl.p,
-                  nullptr, nullptr, &counts, disc->early_exit != 0, nullptr, true);
-    if (rc) return rc;
     int64_t cu = 0;
-    for (auto x : counts) cu += (int64_t)x;
     int32_t jstar = INT32_MAX;
-    CUDA_TRY(ctx, d2h(ctx, &jstar, ctx->jl.p, sizeof(int32_t)));
-    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    // evaluate a list of candidates (ascending), smallest feasible index -> jstar
+    auto sweep = [&](const std::vector<JobSpec> &js, bool early, double *ms_acc, double *kern_acc,
+                     int64_t *eff_acc, int64_t *useful_acc) -> int {
+        int r = fill_int_max(ctx, (int32_t *)ctx->jl.p, 1);
+        if (r) return r;
+        std::vector<uint64_t> counts;
+        r = run_jobs(ctx, cs, cd, disc, js, (int32_t *)ctx->jl.p, nullptr, nullptr, &counts, early, nullptr,
+                     true);
+        if (r) return r;
+        for (auto x : counts) cu += (int64_t)x;
+        *ms_acc += ctx->sweep_ms; *kern_acc += ctx->step_ms;
+        *eff_acc += ctx->last_effective; *useful_acc += ctx->last_useful;
+        int32_t j = INT32_MAX;
+        CUDA_TRY(ctx, d2h(ctx, &j, ctx->jl.p, sizeof(int32_t)));
+        CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+        jstar = j;
+        return MADPIPE_OK;
+    };
+    double ms = 0.0, kern = 0.0;
+    int64_t eff = 0, useful = 0;
+    const int n_c = disc->n_periods;
+    if (disc->early_exit == 2 && n_c > 4) {
+        // NEXT row f3, coarse-to-fine: every s-th candidate in ascending order until one is
+        // feasible (J1), then the candidates of the gap (J1-s, J1).  Exact when feasibility is
+        // monotone in the period; early_exit = 1 is exact without that assumption.
+        const int step = std::max(2, (int)std::lround(std::sqrt((double)n_c)));
+        std::vector<JobSpec> coarse;
+        for (int j = 0; j < n_c; j += step) coarse.push_back({0, j});
+        if (coarse.back().j != n_c - 1) coarse.push_back({0, n_c - 1});
+        rc = sweep(coarse, true, &ms, &kern, &eff, &useful);
+        if (rc) return rc;
+        if (jstar != INT32_MAX && jstar > 0) {
+            const int J1 = jstar;
+            std::vector<JobSpec> fine;
+            for (int j = std::max(0, J1 - step + 1); j < J1; j++) fine.push_back({0, j});
+            if (!fine.empty()) {
+                rc = sweep(fine, true, &ms, &kern, &eff, &useful);
+                if (rc) return rc;
+                if (jstar == INT32_MAX) jstar = J1;
+            }
+        }
+    } else {
+        rc = sweep(shard_jobs(0, n_c, 0, 1), disc->early_exit != 0, &ms, &kern, &eff, &useful);
+        if (rc) return rc;
+    }
+    ctx->sweep_ms = ms; ctx->step_ms = kern;
+    ctx->last_cell_updates = cu; ctx->last_effective = eff; ctx->last_useful = useful;
     if (jstar == INT32_MAX) {
         fill_infeasible(out, cu);
         return MADPIPE_INFEASIBLE;

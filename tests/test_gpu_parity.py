@@ -187,3 +187,27 @@ def test_batch_config_sampled(ctx):
         _same_solution(got, ref)
         assert got["cand_index"] == cfg["chains"][i]["oracle_cand_index"]
         _verify(ch, P, M, B, got)
+
+
+def test_coarse_to_fine_matches_full_sweep_when_monotone(ctx):
+    """NEXT row f3 (early_exit=2): equal to the full sweep whenever feasibility is monotone
+    in the period; checked on fuzz cases and on the CNN configs."""
+    n_checked = 0
+    for ch, P, M, beta, n_m, n_v, n_c, vr in _fuzz_cases(60, 10):
+        n_c = 40
+        tau, root = ctx.candidates(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
+        feas = [root[j] <= tau[j] for j in range(n_c)]
+        if any(feas[j] and not feas[j + 1] for j in range(n_c - 1)):
+            continue            # not monotone: f3 is allowed to differ
+        full = ctx.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
+        ctf = ctx.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr, early_exit=2)
+        _same_solution(ctf, full)
+        n_checked += 1
+    assert n_checked > 30
+    for name in ("resnet50", "vgg19"):
+        cfg = configs.load(name)
+        ch = chaingen.make(cfg["chain"])
+        full = ctx.solve(ch, *_args(cfg), early_exit=True)
+        ctf = ctx.solve(ch, *_args(cfg), early_exit=2)
+        _same_solution(ctf, full)
+        assert ctf["cell_updates"] <= full["cell_updates"] * 2
