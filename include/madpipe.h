@@ -213,6 +213,24 @@ int madpipe_schedule(const madpipe_chain *chain, double beta, double period, int
                      const int32_t *stage_first, const int32_t *stage_last, madpipe_op *ops,
                      int32_t *n_ops);
 
+/* ---- NEXT row f1: the paper-literal MadPipe-DP and Algorithm 1 --------------
+ * The serial baseline the candidate sweep replaces: K = 10 calls
+ * of the optimisation-form DP T(l, p, t_P, m_P, V) with
+ * t_P discretised into n_tp levels on [0, U(1,L)] (101), m_P into n_mem
+ * and V into n_delay levels (PAPER range), driven by the modified binary search
+ * of Algorithm 1 (reading Q15).  out->period = min_i max(T_i, That_i)
+ * (P:199), out->cand_index = that i, the stages come from a device traceback of
+ * DP(That_i) (tie-break Q11); T_hist / That_hist [host, K] (may be NULL) get
+ * every iteration.  cell_updates is 0 (not a sweep).  [host] chain. */
+int madpipe_solve_paper(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M, double beta,
+                        int32_t n_mem, int32_t n_delay, int32_t n_tp, int32_t K, madpipe_alloc *out,
+                        double *T_hist, double *That_hist);
+/* The literal DP table at target That: A_out[(L+1)*P*n_tp*n_delay*n_mem] in
+ * [l][p][t][v][m] order and its decisions (may be NULL), for parity tests. */
+int madpipe_literal_table(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M, double beta,
+                          int32_t n_mem, int32_t n_delay, int32_t n_tp, double That, double *A_out,
+                          int32_t *arg_out);
+
 #ifdef __cplusplus
 }
 #endif

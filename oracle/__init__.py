@@ -81,6 +81,12 @@ def lib():
             L.oracle_solve.argtypes = [cint, dp, dp, ip, ip, cint, ctypes.c_int64, ctypes.c_double,
                                        cint, cint, cint, cint, cint, cint, cint, cint,
                                        dp, dp, dp, dp, dp, i32p, i32p, i32p, i32p, i32p, ip]
+            L.oracle_literal_table.restype = cint
+            L.oracle_literal_table.argtypes = [cint, dp, dp, ip, ip, cint, ctypes.c_int64, ctypes.c_double,
+                                               cint, cint, cint, ctypes.c_double, dp, i32p]
+            L.oracle_literal_solve.restype = cint
+            L.oracle_literal_solve.argtypes = [cint, dp, dp, ip, ip, cint, ctypes.c_int64, ctypes.c_double,
+                                               cint, cint, cint, cint, dp, dp, dp, i32p, i32p, i32p, i32p, i32p]
             _lib = L
     return _lib
 
@@ -176,3 +182,33 @@ def solve(ch, P, M, beta, n_m, n_v, n_c, v_range=PAPER, early_exit=False, j_lo=0
                 cand_index=ci.value,
                 stages=[(int(sf[i]), int(sl_[i]), int(sp[i])) for i in range(n)],
                 cell_updates=cu.value, tau=tau, root=root)
+
+
+def literal_table(ch, P, M, beta, n_m, n_v, n_t, That, with_arg=True):
+    """NEXT row f1: the paper-literal DP table T(l, p, t, v, m) at target That (layout
+    [l][p][t][v][m]) and its decisions."""
+    L, keep, ptrs = _chain_args(ch)
+    A = np.empty((L + 1, P, n_t, n_v, n_m), np.float64)
+    ARG = np.empty((L + 1, P, n_t, n_v, n_m), np.int32) if with_arg else None
+    rc = lib().oracle_literal_table(L, *ptrs, P, M, beta, n_m, n_v, n_t, That, _ptr(A, ctypes.c_double),
+                                    _ptr(ARG, ctypes.c_int32) if with_arg else None)
+    if rc:
+        raise ValueError("oracle_literal_table rc=%d" % rc)
+    return A, ARG
+
+
+def literal_solve(ch, P, M, beta, n_m, n_v, n_t, K=10):
+    """NEXT row f1: Algorithm 1 (reading Q15) around the literal DP."""
+    L, keep, ptrs = _chain_args(ch)
+    T = np.empty(K); Th = np.empty(K)
+    period = ctypes.c_double(); bi = ctypes.c_int32(); ns = ctypes.c_int32()
+    sf = np.zeros(L, np.int32); sl = np.zeros(L, np.int32); sp = np.zeros(L, np.int32)
+    rc = lib().oracle_literal_solve(L, *ptrs, P, M, beta, n_m, n_v, n_t, K, _ptr(T, ctypes.c_double),
+                                    _ptr(Th, ctypes.c_double), ctypes.byref(period), ctypes.byref(bi),
+                                    ctypes.byref(ns), _ptr(sf, ctypes.c_int32), _ptr(sl, ctypes.c_int32),
+                                    _ptr(sp, ctypes.c_int32))
+    if rc < 0:
+        raise ValueError("oracle_literal_solve rc=%d" % rc)
+    n = ns.value
+    return dict(rc=rc, T=T, That=Th, period=period.value, best_iter=bi.value,
+                stages=[(int(sf[i]), int(sl[i]), int(sp[i])) for i in range(n)])

@@ -192,3 +192,63 @@ def value_of_stages(ch, P, M, beta, n_m, n_v, v_range, tau, stages):
     c = Chain(ch, P, M, beta, n_m, n_v, v_range)
     alloc = [((f, l), 1 if pr == P - 1 else 0) for (f, l, pr) in stages]
     return evaluate(c, tau, alloc, P - 1, 0, 0, True)
+
+
+# --------------------------------------------------------------------------
+# NEXT row f1: the paper-literal optimisation form (t_P discretised)
+# --------------------------------------------------------------------------
+def literal_evaluate(c: Chain, That, n_t, alloc, p, t, m, v):
+    """Period the literal DP assigns to `alloc` (chain order) of layers 1..l from
+    state (p, t, m, v): the max of every term met along the path -- normal stage
+    loads U(k,l), boundary times C(k-1), the special load t*dt after each special
+    stage (each stage's load rounded up to the t grid), U(1,l) + t*dt at the p = 0
+    base, t*dt at l = 0.  INF if a constraint fails."""
+    n_m, M = c.n_m, c.M
+    dV = c.vmax(That) / float(c.n_v - 1)
+    dt = c.Up[c.L] / float(n_t - 1)
+    V = float(v) * dV
+    terms = []
+    for idx in range(len(alloc) - 1, -1, -1):
+        (k, l), o = alloc[idx]
+        Ukl = c.U(k, l)
+        g = math.ceil((V + Ukl) / That)
+        if p == 0:                                   # base: the single remaining stage 1..l
+            D = c.mem(k, l, g - 1)
+            if k != 1 or o != 1 or m + -(-(D * (n_m - 1)) // M) > n_m - 1:
+                return INF
+            terms.append(Ukl + float(t) * dt)
+            return max(terms)
+        if k > 1:
+            terms.append(c.C[k - 1])
+        if o == 0:
+            if c.mem(k, l, g) > M:
+                return INF
+            terms.append(Ukl)
+            p -= 1
+        else:
+            D = c.mem(k, l, g - 1)
+            dd = -(-(D * (n_m - 1)) // M)
+            ts = math.ceil(Ukl / dt)
+            if m + dd > n_m - 1 or t + ts > n_t - 1:
+                return INF
+            m += dd
+            t += ts
+            terms.append(float(t) * dt)
+        if k > 1:
+            Vn = oplus(oplus(V, Ukl, That), c.C[k - 1], That)
+            q = math.ceil(Vn / dV)
+            if q > c.n_v - 1:
+                return INF
+            V = float(q) * dV
+    terms.append(float(t) * dt)                        # T(0, p, t_P, ...) = t_P
+    return max(terms)
+
+
+def literal_root(ch, P, M, beta, n_m, n_v, n_t, That):
+    c = Chain(ch, P, M, beta, n_m, n_v, 0)
+    best = INF
+    for alloc in allocations(c.L, P - 1):
+        val = literal_evaluate(c, That, n_t, alloc, P - 1, 0, 0, 0)
+        if val < best:
+            best = val
+    return best

@@ -455,3 +455,162 @@ int oracle_solve(int L, const double *uF, const double *uB, const int64_t *W, co
     chain_free(&c);
     return OR_OK;
 }
+
+/* ====================================================================
+ * NEXT row f1: the paper-literal MadPipe-DP and Algorithm 1.
+ *
+ * T(l, p, t_P, m_P, V) of P:173 as a period (optimisation form), with t_P a
+ * discretised state (n_t values in [0, U(1,L)]), for a fixed target
+ * T-hat that drives the 1F1B* memory estimate (g, (+)):
+ *   N: max(U(k,l), C(k-1), T(k-1, p-1, t, m, v'))   if M(k,l,g) <= M
+ *   S: max(t'dt, C(k-1), T(k-1, p, t', m+d, v'))    if m+d <= n_m-1
+ *              with t' = t + ceil(U(k,l)/dt) (reading L1: each special stage's
+ *              load is rounded up to the t grid), infeasible if t' > n_t-1
+ *   T(0,p,t,..) = t dt;  T(l,0,t,m,v) = U(1,l) + t dt if m + d(1,l,v) <= n_m-1
+ *   T = min over k of the above, tie-break Q11; root T(L,P-1,0,0,0).
+ * No tau-window here: any k is allowed, the period just grows.
+ * Layout A[l][p][t][v][m].
+ * ==================================================================== */
+#define LIDX(c, nt, l, p, t, v, m) \
+    (((((size_t)(l) * (size_t)(c)->P + (size_t)(p)) * (size_t)(nt) + (size_t)(t)) * (size_t)(c)->n_v + \
+      (size_t)(v)) * (size_t)(c)->n_m + (size_t)(m))
+
+static double dmax(double a, double b) { return a > b ? a : b; }
+
+static int64_t literal_fill(const chain_t *c, double That, int n_t, double *A, int32_t *ARG)
+{
+    const int L = c->L, P = c->P, n_v = c->n_v, n_m = c->n_m;
+    const double dV = v_max(c, That) / (double)(n_v - 1);
+    const double dt = c->Up[L] / (double)(n_t - 1);
+    int64_t updates = 0;
+    for (int p = 0; p < P; p++)
+        for (int t = 0; t < n_t; t++)
+            for (int v = 0; v < n_v; v++)
+                for (int m = 0; m < n_m; m++) {
+                    A[LIDX(c, n_t, 0, p, t, v, m)] = (double)t * dt;     /* T(0,p,t_P,..) = t_P */
+                    if (ARG) ARG[LIDX(c, n_t, 0, p, t, v, m)] = -1;
+                }
+    for (int l = 1; l <= L; l++) {
+        double U1l = U(c, 1, l);
+        for (int v = 0; v < n_v; v++) {
+            trans_t tb = transition(c, That, dV, 1, l, v);
+            for (int t = 0; t < n_t; t++)
+                for (int m = 0; m < n_m; m++) {
+                    int ok = (int64_t)m + tb.d <= (int64_t)(n_m - 1);
+                    A[LIDX(c, n_t, l, 0, t, v, m)] = ok ? U1l + (double)t * dt : INFINITY;
+                    if (ARG) ARG[LIDX(c, n_t, l, 0, t, v, m)] = ok ? 3 : -1;
+                }
+        }
+        if (P > 1) updates += (int64_t)l * (P - 1) * n_t * n_v * n_m;
+        for (int v = 0; v < n_v; v++) {
+            for (int p = 1; p < P; p++)
+                for (int t = 0; t < n_t; t++)
+                    for (int m = 0; m < n_m; m++) {
+                        A[LIDX(c, n_t, l, p, t, v, m)] = INFINITY;
+                        if (ARG) ARG[LIDX(c, n_t, l, p, t, v, m)] = -1;
+                    }
+            for (int k = 1; k <= l; k++) {
+                trans_t tr = transition(c, That, dV, k, l, v);
+                if (k > 1 && tr.vn == VN_OVERFLOW) continue;
+                double Ukl = U(c, k, l);
+                double Ck = k > 1 ? c->C[k - 1] : 0.0;
+                int64_t dts = (int64_t)ceil(Ukl / dt);
+                for (int p = 1; p < P; p++)
+                    for (int t = 0; t < n_t; t++)
+                        for (int m = 0; m < n_m; m++) {
+                            double *best = &A[LIDX(c, n_t, l, p, t, v, m)];
+                            if (tr.nf) {                                   /* T_N */
+                                double cand = dmax(dmax(Ukl, Ck), A[LIDX(c, n_t, k - 1, p - 1, t, tr.vn, m)]);
+                                if (cand < *best) { *best = cand; if (ARG) ARG[LIDX(c, n_t, l, p, t, v, m)] = 2 * k; }
+                            }
+                            if ((int64_t)m + tr.d <= (int64_t)(n_m - 1) && (int64_t)t + dts <= (int64_t)(n_t - 1)) {
+                                int t2 = t + (int)dts;                     /* T_S */
+                                double cand = dmax(dmax((double)t2 * dt, Ck),
+                                                   A[LIDX(c, n_t, k - 1, p, t2, tr.vn, m + (int)tr.d)]);
+                                if (cand < *best) { *best = cand; if (ARG) ARG[LIDX(c, n_t, l, p, t, v, m)] = 2 * k + 1; }
+                            }
+                        }
+            }
+        }
+    }
+    return updates;
+}
+
+int oracle_literal_table(int L, const double *uF, const double *uB, const int64_t *W, const int64_t *a,
+                         int P, int64_t M, double beta, int n_m, int n_v, int n_t, double That,
+                         double *A_out, int32_t *arg_out)
+{
+    chain_t c;
+    int rc = chain_init(&c, L, uF, uB, W, a, P, M, beta, n_m, n_v, VR_PAPER);
+    if (rc || n_t < 2 || !(That > 0.0)) { chain_free(&c); return rc ? rc : OR_EINVAL; }
+    literal_fill(&c, That, n_t, A_out, arg_out);
+    chain_free(&c);
+    return OR_OK;
+}
+
+/* Algorithm 1 (reading Q15): K calls of the literal DP; returns the
+ * best max(T_i, That_i), its index and allocation (traceback of that call). */
+int oracle_literal_solve(int L, const double *uF, const double *uB, const int64_t *W, const int64_t *a,
+                         int P, int64_t M, double beta, int n_m, int n_v, int n_t, int K,
+                         double *T_hist, double *That_hist, double *period, int *best_iter,
+                         int *n_stages, int *stage_first, int *stage_last, int *stage_proc)
+{
+    chain_t c;
+    int rc = chain_init(&c, L, uF, uB, W, a, P, M, beta, n_m, n_v, VR_PAPER);
+    if (rc || n_t < 2 || K < 1) { chain_free(&c); return rc ? rc : OR_EINVAL; }
+    size_t cells = (size_t)(L + 1) * (size_t)P * (size_t)n_t * (size_t)n_v * (size_t)n_m;
+    double *A = (double *)malloc(sizeof(double) * cells);
+    int32_t *ARG = (int32_t *)malloc(sizeof(int32_t) * cells);
+    if (!A || !ARG) { free(A); free(ARG); chain_free(&c); return OR_ENOMEM; }
+    double lb = c.Up[L] / (double)P;                  /* line 1 */
+    double ub = c.Up[L] + c.SC;                       /* line 2 (Q4) */
+    double That = lb;                                 /* line 3 */
+    double best = INFINITY;
+    int bi = -1;
+    for (int i = 0; i < K; i++) {
+        literal_fill(&c, That, n_t, A, NULL);
+        double T = A[LIDX(&c, n_t, L, P - 1, 0, 0, 0)];   /* T_i = MadPipe-DP(That_i) */
+        T_hist[i] = T; That_hist[i] = That;
+        double Tm = T > That ? T : That;                   /* max(T_i, That_i) */
+        if (Tm < best) { best = Tm; bi = i; }
+        double lo = T < That ? T : That;
+        if (lo > lb) lb = lo;                              /* lb <- max(lb, min(T, That)) */
+        if (Tm < ub) ub = Tm;                              /* ub <- min(ub, max(T, That)) */
+        That = (lb + ub) / 2.0;
+    }
+    *period = best;
+    *best_iter = bi;
+    *n_stages = 0;
+    if (bi >= 0 && isfinite(best)) {
+        double Tb = That_hist[bi];
+        literal_fill(&c, Tb, n_t, A, ARG);
+        const double dV = v_max(&c, Tb) / (double)(n_v - 1);
+        const double dt = c.Up[L] / (double)(n_t - 1);
+        int l = L, p = P - 1, t = 0, v = 0, m = 0, ns = 0;
+        int *kind = (int *)malloc(sizeof(int) * (size_t)L);
+        while (l > 0) {
+            if (p == 0) { stage_first[ns] = 1; stage_last[ns] = l; kind[ns] = 1; ns++; break; }
+            int32_t arg = ARG[LIDX(&c, n_t, l, p, t, v, m)];
+            if (arg < 0) break;
+            int k = arg >> 1, o = arg & 1;
+            trans_t tr = transition(&c, Tb, dV, k, l, v);
+            stage_first[ns] = k; stage_last[ns] = l; kind[ns] = o; ns++;
+            if (o) { m += (int)tr.d; t += (int)(int64_t)ceil(U(&c, k, l) / dt); } else p -= 1;
+            v = tr.vn;
+            l = k - 1;
+        }
+        for (int i = 0; i < ns / 2; i++) {
+            int j = ns - 1 - i, tmp;
+            tmp = stage_first[i]; stage_first[i] = stage_first[j]; stage_first[j] = tmp;
+            tmp = stage_last[i]; stage_last[i] = stage_last[j]; stage_last[j] = tmp;
+            tmp = kind[i]; kind[i] = kind[j]; kind[j] = tmp;
+        }
+        int next_normal = 0;
+        for (int i = 0; i < ns; i++) stage_proc[i] = kind[i] ? P - 1 : next_normal++;
+        *n_stages = ns;
+        free(kind);
+    }
+    free(A); free(ARG);
+    chain_free(&c);
+    return isfinite(best) ? OR_OK : OR_INFEASIBLE;
+}

@@ -195,6 +195,30 @@ class Context:
                 self.h)
         return A, ARG
 
+    # ------------------------------------------------------------------ NEXT row f1
+    def solve_paper(self, chain, P, M, beta, n_mem=11, n_delay=51, n_tp=101, K=10):
+        """Paper-literal MadPipe-DP + Algorithm 1 (P:173-205, P:233 discretisation)."""
+        hc = N.HostChain(chain)
+        buf = N.AllocBuf(hc.L)
+        T = np.empty(K); Th = np.empty(K)
+        rc = self._lib.madpipe_solve_paper(self.h, ctypes.byref(hc.c), int(P), int(M), float(beta), int(n_mem),
+                                           int(n_delay), int(n_tp), int(K), ctypes.byref(buf.s),
+                                           T.ctypes.data_as(N._dp), Th.ctypes.data_as(N._dp))
+        N.check(rc, self.h)
+        r = buf.result(rc)
+        r.update(T=T, That=Th, best_iter=r["cand_index"])
+        return r
+
+    def literal_table(self, chain, P, M, beta, n_mem, n_delay, n_tp, That, with_arg=True):
+        hc = N.HostChain(chain)
+        A = np.empty((hc.L + 1, P, n_tp, n_delay, n_mem), np.float64)
+        ARG = np.empty(A.shape, np.int32) if with_arg else None
+        N.check(self._lib.madpipe_literal_table(self.h, ctypes.byref(hc.c), int(P), int(M), float(beta),
+                                                int(n_mem), int(n_delay), int(n_tp), float(That),
+                                                A.ctypes.data_as(N._dp),
+                                                ARG.ctypes.data_as(N._i32p) if with_arg else None), self.h)
+        return A, ARG
+
     def set_timing(self, per_launch: bool):
         N.check(self._lib.madpipe_set_timing(self.h, 1 if per_launch else 0), self.h)
 

@@ -399,7 +399,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         size_t used = 0;
         int maxL = 0;
         size_t max_slab = 0;
-        int smem_tma = 0, stage_doubles = 0;
+        int smem_tma = 0;
         for (; next < js.size(); next++) {
             const JobSpec &s = js[next];
             if (early_exit && jl_host[s.chain] < s.j) continue;
@@ -946,5 +946,155 @@ extern "C" int madpipe_dp_table(madpipe_ctx *ctx, const madpipe_chain *chain, in
     if (arg_out)
         CUDA_TRY(ctx, d2h(ctx, arg_out, hook.arg_dev, cells * sizeof(int32_t)));
     CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    return MADPIPE_OK;
+}
+
+// ---------------------------------------------------------------------------
+// NEXT row f1: paper-literal MadPipe-DP + Algorithm 1 (mp_literal.cu)
+// ---------------------------------------------------------------------------
+namespace {
+
+struct LitRun {
+    std::vector<ChainSpec> cs;
+    std::vector<ChainDev> cd;
+    Job hj{};
+    Job *dj = nullptr;
+    int nmp = 2, n_t = 2;
+    double dt = 0.0, U = 0.0, SC = 0.0, lb = 0.0, ub = 0.0;
+    size_t cells = 0;
+};
+
+int lit_setup(madpipe_ctx *ctx, LitRun &R, const madpipe_chain *chain, int32_t P, int64_t M, double beta,
+              int n_mem, int n_delay, int n_t) {
+    madpipe_disc d{n_mem, n_delay, 1, MADPIPE_VRANGE_PAPER, 0};
+    int rc = check_one(ctx, chain, P, M, beta, &d, true);
+    if (rc) return rc;
+    if (n_t < 2 || n_t > 1 << 20) return fail(ctx, MADPIPE_EINVAL, "n_tp must be in [2, 2^20]");
+    R.cs = {{*chain, false, P, M, beta}};
+    rc = upload_chains(ctx, R.cs, R.cd);
+    if (rc) return rc;
+    double scal[4];
+    CUDA_TRY(ctx, d2h(ctx, scal, R.cd[0].scal, sizeof scal));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    R.SC = scal[0]; R.lb = scal[1]; R.ub = scal[2]; R.U = scal[3];
+    R.n_t = n_t;
+    R.dt = R.U / (double)(n_t - 1);              // n_t values in [0, U(1,L)]
+    R.nmp = nmp_of(n_mem);
+    R.cells = (size_t)(chain->L + 1) * n_delay * (size_t)n_t * P * R.nmp;
+    CUDA_TRY(ctx, ctx->tables.ensure(R.cells * sizeof(double)));
+    CUDA_TRY(ctx, ctx->jobs.ensure(sizeof(Job)));
+    Job &J = R.hj;
+    const ChainDev &c = R.cd[0];
+    J.Up = c.Up; J.Wp = c.Wp; J.Ap = c.Ap; J.a = c.a; J.C = c.C; J.scal = c.scal;
+    J.table = (double *)ctx->tables.p;
+    J.M = M; J.L = chain->L; J.P = P; J.n_v = n_delay; J.n_m = n_mem; J.vsafe = 0;
+    J.dV = (R.U + R.SC) / (double)(n_delay - 1);  // PAPER V range (Q8)
+    R.dj = (Job *)ctx->jobs.p;
+    return MADPIPE_OK;
+}
+
+// one literal DP at target That; returns its root T(L, P-1, 0, 0, 0)
+int lit_run(madpipe_ctx *ctx, LitRun &R, double That, double *root) {
+    R.hj.tau = That;
+    CUDA_TRY(ctx, h2d(ctx, R.dj, &R.hj, sizeof(Job)));
+    launch_lit_init(R.dj, R.n_t, R.dt, R.nmp, (int64_t)R.hj.n_v * R.n_t * R.hj.P * R.nmp, ctx->stream);
+    for (int l = 1; l <= R.hj.L; l++)
+        launch_lit_step(R.dj, R.n_t, R.dt, R.nmp, R.hj.n_v, R.hj.P, l, ctx->stream);
+    ctx->launches += 1 + R.hj.L;
+    CUDA_TRY(ctx, cudaGetLastError());
+    const size_t ridx = (((size_t)R.hj.L * R.hj.n_v) * R.n_t * (size_t)R.hj.P + (size_t)(R.hj.P - 1)) * R.nmp;
+    CUDA_TRY(ctx, d2h(ctx, root, (double *)ctx->tables.p + ridx, sizeof(double)));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    return MADPIPE_OK;
+}
+
+}  // namespace
+
+extern "C" int madpipe_literal_table(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                                     double beta, int32_t n_mem, int32_t n_delay, int32_t n_tp, double That,
+                                     double *A_out, int32_t *arg_out) {
+    int rc = begin(ctx);
+    if (rc) return rc;
+    if (!A_out || !(That > 0.0)) return fail(ctx, MADPIPE_EINVAL, "bad A_out / That");
+    LitRun R;
+    rc = lit_setup(ctx, R, chain, P, M, beta, n_mem, n_delay, n_tp);
+    if (rc) return rc;
+    double root;
+    rc = lit_run(ctx, R, That, &root);
+    if (rc) return rc;
+    const size_t out_cells = (size_t)(chain->L + 1) * P * n_tp * n_delay * n_mem;
+    CUDA_TRY(ctx, ctx->scratch.ensure(out_cells * (sizeof(double) + sizeof(int32_t))));
+    double *A_dev = (double *)ctx->scratch.p;
+    int32_t *arg_dev = (int32_t *)(A_dev + out_cells);
+    launch_lit_export(R.dj, R.n_t, R.dt, R.nmp, A_dev, arg_out ? arg_dev : nullptr, ctx->stream);
+    CUDA_TRY(ctx, cudaGetLastError());
+    CUDA_TRY(ctx, d2h(ctx, A_out, A_dev, out_cells * sizeof(double)));
+    if (arg_out) CUDA_TRY(ctx, d2h(ctx, arg_out, arg_dev, out_cells * sizeof(int32_t)));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    return MADPIPE_OK;
+}
+
+extern "C" int madpipe_solve_paper(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
+                                   double beta, int32_t n_mem, int32_t n_delay, int32_t n_tp, int32_t K,
+                                   madpipe_alloc *out, double *T_hist, double *That_hist) {
+    int rc = begin(ctx);
+    if (rc) return rc;
+    if (!out || K < 1) return fail(ctx, MADPIPE_EINVAL, "bad out / K");
+    LitRun R;
+    rc = lit_setup(ctx, R, chain, P, M, beta, n_mem, n_delay, n_tp);
+    if (rc) return rc;
+    double lb = R.lb, ub = R.ub, That = lb;   // Algorithm 1 lines 1-3 (Q4)
+    double best = INFINITY, best_That = 0.0;
+    int bi = -1;
+    for (int i = 0; i < K; i++) {
+        double T;
+        rc = lit_run(ctx, R, That, &T);           // line 4: T_i = MadPipe-DP(That_i)
+        if (rc) return rc;
+        if (T_hist) T_hist[i] = T;
+        if (That_hist) That_hist[i] = That;
+        const double Tm = T > That ? T : That;    // max(T_i, That_i)
+        if (Tm < best) { best = Tm; bi = i; best_That = That; }
+        const double lo = T < That ? T : That;
+        if (lo > lb) lb = lo;                     // lb <- max(lb, min(T_i, That_i))  (Q15)
+        if (Tm < ub) ub = Tm;                     // ub <- min(ub, max(T_i, That_i))
+        That = (lb + ub) / 2.0;
+    }
+    fill_infeasible(out, 0);
+    if (bi < 0 || !std::isfinite(best)) return MADPIPE_INFEASIBLE;
+    double root;
+    rc = lit_run(ctx, R, best_That, &root);       // re-solve the winner and trace it back
+    if (rc) return rc;
+    const int L = chain->L;
+    CUDA_TRY(ctx, ctx->stages.ensure(sizeof(int32_t) * (3 * (size_t)L + 1)));
+    int32_t *st = (int32_t *)ctx->stages.p;
+    launch_lit_traceback(R.dj, R.n_t, R.dt, R.nmp, st, st + 3 * L, ctx->stream);
+    ctx->launches++;
+    CUDA_TRY(ctx, cudaGetLastError());
+    std::vector<int32_t> h(3 * (size_t)L + 1);
+    CUDA_TRY(ctx, d2h(ctx, h.data(), st, h.size() * sizeof(int32_t)));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    const int ns = h[3 * L];
+    if (ns < 0) return fail(ctx, MADPIPE_ESTATE, "literal traceback found no decision");
+    // reverse into chain order, number the normal GPUs, allocation period
+    std::vector<double> Up(L + 1, 0.0);
+    for (int i = 1; i <= L; i++) Up[i] = Up[i - 1] + (chain->uF[i - 1] + chain->uB[i - 1]);
+    int next_normal = 0;
+    double lp = 0.0, special = 0.0;
+    for (int q = 0; q < ns; q++) {
+        const int src = ns - 1 - q;
+        const int f = h[src], l = h[L + src], kind = h[2 * L + src];
+        const double u = Up[l] - Up[f - 1];
+        if (out->stage_first) out->stage_first[q] = f;
+        if (out->stage_last) out->stage_last[q] = l;
+        if (out->stage_proc) out->stage_proc[q] = kind ? P - 1 : next_normal;
+        if (!kind) { next_normal++; lp = std::max(lp, u); } else special += u;
+        if (f > 1) lp = std::max(lp, 2.0 * (double)chain->a[f - 1] / beta);
+    }
+    out->n_stages = ns;
+    out->period = best;
+    out->special_load = special;
+    out->load_period = std::max(lp, special);
+    out->cand_index = bi;
+    out->cell_updates = 0;
     return MADPIPE_OK;
 }

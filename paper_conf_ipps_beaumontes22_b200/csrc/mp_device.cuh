@@ -37,8 +37,10 @@ constexpr int32_t kSkip = (int32_t)0x80000000;
 // g = ceil((V + U(k,l)) / tau); nf = M(k,l,g) <= M; d = ceil(M(k,l,g-1)(n_m-1)/M)
 // (reading Q7); for k > 1 the next delay V' = (V (+) U) (+) C(k-1) rounded up to
 // the grid (readings Q2, Q6, Q8).  Returns kSkip if neither option is possible.
+// skip_comm = false is the optimisation form of NEXT row f1 (mp_literal.cu),
+// where a communication longer than T-hat is not a skip: it enters the max.
 __device__ __forceinline__ int32_t transition(const Job &J, int k, int l, int v, double Ukl,
-                                              int64_t *d_out) {
+                                              int64_t *d_out, bool skip_comm = true) {
     const double V = __dmul_rn((double)v, J.dV);
     const int64_t g = (int64_t)ceil(__ddiv_rn(__dadd_rn(V, Ukl), J.tau));
     const bool nf = mem_kl(J, k, l, g) <= J.M;
@@ -48,7 +50,7 @@ __device__ __forceinline__ int32_t transition(const Job &J, int k, int l, int v,
     int vn = 0;
     if (k > 1) {
         const double ck = J.C[k - 1];
-        if (ck > J.tau) return kSkip;
+        if (skip_comm && ck > J.tau) return kSkip;
         const double Vn = oplus(oplus(V, Ukl, J.tau), ck, J.tau);
         const double q = ceil(__ddiv_rn(Vn, J.dV));
         if (q > (double)(J.n_v - 1)) {

@@ -97,6 +97,12 @@ void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int 
 int persist_nsg(int np, int vb, int nmp);
 void tma_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
 void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, cudaStream_t s);
+void launch_lit_init(const Job *job, int n_t, double dt, int nmp, int64_t cells, cudaStream_t s);
+void launch_lit_step(const Job *job, int n_t, double dt, int nmp, int n_v, int P, int l, cudaStream_t s);
+void launch_lit_export(const Job *job, int n_t, double dt, int nmp, double *A_out, int32_t *arg_out,
+                       cudaStream_t s);
+void launch_lit_traceback(const Job *job, int n_t, double dt, int nmp, int32_t *stages, int32_t *n_out,
+                          cudaStream_t s);
 void launch_root(const Job *jobs, int n_jobs, int nmp, int32_t *jl_per_chain, double *root_out,
                  double *tau_out, cudaStream_t s);
 void launch_count(const Job *jobs, int n_jobs, unsigned long long *counts, cudaStream_t s);

@@ -27,10 +27,10 @@ __global__ void prep_kernel(ChainDev *chains) {
     __shared__ double s_u[CH];
     __shared__ int64_t s_w[CH];
     __shared__ int64_t s_a[CH];
-    __shared__ double s_up, s_sc;
+    __shared__ double s_up;
     __shared__ int64_t s_wp, s_ap;
     if (threadIdx.x == 0) {
-        s_up = 0.0; s_wp = 0; s_ap = 0; s_sc = 0.0;
+        s_up = 0.0; s_wp = 0; s_ap = 0;
         c.Up[0] = 0.0; c.Wp[0] = 0; c.Ap[0] = 0; c.C[0] = 0.0;
     }
     for (int base = 1; base <= L; base += CH) {
