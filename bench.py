@@ -181,6 +181,8 @@ def main():
     dev = torch.device("cuda", local)
     use_dist = world > 1 or args.force_dist
     if use_dist:
+        if os.environ.get("NCCL_DEBUG", "VERSION").upper() == "VERSION":
+            os.environ["NCCL_DEBUG"] = "WARN"      # keep stdout to the one JSON line
         dist.init_process_group("nccl", device_id=dev)
     stream = torch.cuda.current_stream(dev)
     ctx = mp.Context(local, stream=stream.cuda_stream)
