@@ -50,7 +50,7 @@ struct Job {
     unsigned long long *useful;  // live relaxations whose source row is not all +inf
     struct TransEntry *tlist;    // [n_v][code_cap] useful transitions of layer l (persist path)
     int32_t *tcount;             // [n_v] their number
-    int32_t pad2_[2];
+    int32_t *kwin;               // [L+1] window start max(kmin_tau(l), kmin_W(l)) (window_kernel)
 };
 
 // One useful transition of layer l for delay row v, in ascending k (trans_kernel).
@@ -97,6 +97,7 @@ void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int 
 int persist_nsg(int np, int vb, int nmp);
 void tma_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
 void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, cudaStream_t s);
+void launch_window(const Job *jobs, int n_jobs, int max_L, cudaStream_t s);
 void launch_lit_init(const Job *job, int n_t, double dt, int nmp, int64_t cells, cudaStream_t s);
 void launch_lit_step(const Job *job, int n_t, double dt, int nmp, int n_v, int P, int l, cudaStream_t s);
 void launch_lit_export(const Job *job, int n_t, double dt, int nmp, double *A_out, int32_t *arg_out,

@@ -284,7 +284,7 @@ __global__ void __launch_bounds__(256) trans_kernel(const Job *jobs, int l, int 
             o[m] = (m < J.n_m && U1l <= J.tau && (int64_t)m + d <= (int64_t)(J.n_m - 1)) ? U1l : MP_INF;
         if (lane == 0) J.rowflag[(size_t)l * J.n_v + v] = ok ? 1u : 0u;
     }
-    const int kmin = max(kmin_of(J, l), kmin_mem(J, l));
+    const int kmin = J.kwin[l];   // max(kmin_tau(l), kmin_W(l)), precomputed by window_kernel
     unsigned live = 0, useful = 0;
     int n = 0;
     TransEntry *list = J.tlist + (size_t)v * J.code_cap;
@@ -321,6 +321,22 @@ __global__ void __launch_bounds__(256) trans_kernel(const Job *jobs, int l, int 
         atomicAdd(J.eff, (unsigned long long)live * per);
         if (useful) atomicAdd(J.useful, (unsigned long long)useful * per);
     }
+}
+
+// window start of every layer of every job (the binary searches are the same for
+// all delay rows of a job, so they run once per batch instead of once per row)
+__global__ void window_kernel(const Job *jobs, int n_jobs, int max_L) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    const int job = i / max_L, l = 1 + i - (i / max_L) * max_L;
+    if (job >= n_jobs) return;
+    const Job &J = jobs[job];
+    if (l > J.L) return;
+    J.kwin[l] = max(kmin_of(J, l), kmin_mem(J, l));
+}
+
+void launch_window(const Job *jobs, int n_jobs, int max_L, cudaStream_t s) {
+    const int n = n_jobs * max_L;
+    window_kernel<<<(n + 255) / 256, 256, 0, s>>>(jobs, n_jobs, max_L);
 }
 
 void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, cudaStream_t s) {
