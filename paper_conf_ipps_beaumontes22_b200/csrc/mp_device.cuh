@@ -33,6 +33,28 @@ __device__ __forceinline__ double oplus(double x, double y, double tau) {
 
 constexpr int32_t kSkip = (int32_t)0x80000000;
 
+// d = ceil(D (n_m-1) / M) for D >= 0, M > 0 (reading Q7), exactly, without a
+// software int64 division: an fp64 estimate, then a 128-bit check of
+// (d-1) M < D (n_m-1) <= d M and a +-1 correction.  D (n_m-1) + M - 1 fits in
+// int64 (madpipe_validate); only d <= n_m matters to the callers, larger values
+// mean "does not fit", so the result is clamped to n_m+1.
+__device__ __forceinline__ int64_t ceil_div_levels(int64_t D, int nm1, int64_t M) {
+    const uint64_t X = (uint64_t)D * (uint64_t)nm1;
+    if (X == 0) return 0;
+    if (D > M) return nm1 + 2;                       // d > n_m - 1: no level fits
+    int64_t d = (int64_t)ceil(__ddiv_rn((double)X, (double)M));
+    if (d < 1) d = 1;
+    // d*M >= X ?  (128-bit: d <= n_m+1 is small, M < 2^63)
+    auto ge = [&](int64_t q) {
+        const uint64_t lo = (uint64_t)q * (uint64_t)M;
+        const uint64_t hi = __umul64hi((uint64_t)q, (uint64_t)M);
+        return hi > 0 || lo >= X;
+    };
+    while (!ge(d)) d++;
+    while (d > 1 && ge(d - 1)) d--;
+    return d;
+}
+
 // Transition of stage k..l entered with delay level v:
 // g = ceil((V + U(k,l)) / tau); nf = M(k,l,g) <= M; d = ceil(M(k,l,g-1)(n_m-1)/M)
 // (reading Q7); for k > 1 the next delay V' = (V (+) U) (+) C(k-1) rounded up to
@@ -45,7 +67,7 @@ __device__ __forceinline__ int32_t transition(const Job &J, int k, int l, int v,
     const int64_t g = (int64_t)ceil(__ddiv_rn(__dadd_rn(V, Ukl), J.tau));
     const bool nf = mem_kl(J, k, l, g) <= J.M;
     const int64_t D = mem_kl(J, k, l, g - 1);
-    const int64_t d = (D * (int64_t)(J.n_m - 1) + J.M - 1) / J.M;
+    const int64_t d = ceil_div_levels(D, J.n_m - 1, J.M);
     if (d_out) *d_out = d;
     int vn = 0;
     if (k > 1) {
