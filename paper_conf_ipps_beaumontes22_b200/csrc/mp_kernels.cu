@@ -263,9 +263,15 @@ void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, i
 // (a row that is +inf everywhere can only contribute +inf).  Also counts the
 // job's effective and useful relaxations.
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(256) trans_kernel(const Job *jobs, int l, int nmp) {
-    // one warp per delay row v of the job (8 rows per CTA)
-    const Job &J = jobs[blockIdx.y];
+__global__ void __launch_bounds__(256, 4) trans_kernel(const Job *jobs, int l, int nmp) {
+    // one warp per delay row v of the job (8 rows per CTA); the job descriptor is
+    // read once into shared memory (every field access would otherwise be a load)
+    __shared__ Job sJ;
+    if (threadIdx.x < sizeof(Job) / 8)
+        reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
+            __ldg(reinterpret_cast<const uint64_t *>(jobs + blockIdx.y) + threadIdx.x);
+    __syncthreads();
+    const Job &J = sJ;
     if (l > J.L) return;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int v = blockIdx.x * 8 + warp;
