@@ -264,8 +264,9 @@ void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, i
 // job's effective and useful relaxations.
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(256, 4) trans_kernel(const Job *jobs, int l, int nmp) {
-    // one warp per delay row v of the job (8 rows per CTA); the job descriptor is
-    // read once into shared memory (every field access would otherwise be a load)
+    // one half-warp per delay row v of the job (16 rows per CTA: the windows are
+    // short, and the kernel is latency-bound, so fewer, fuller warps win); the job
+    // descriptor is read once into shared memory
     __shared__ Job sJ;
     if (threadIdx.x < sizeof(Job) / 8)
         reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
@@ -274,32 +275,34 @@ __global__ void __launch_bounds__(256, 4) trans_kernel(const Job *jobs, int l, i
     const Job &J = sJ;
     if (l > J.L) return;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int v = blockIdx.x * 8 + warp;
-    if (v >= J.n_v) return;
+    const int half = lane >> 4, hl = lane & 15;
+    const int v = blockIdx.x * 16 + warp * 2 + half;
+    const bool row_ok = v < J.n_v;
+    if (__ballot_sync(0xffffffffu, row_ok) == 0u) return;
     const size_t rowlen = (size_t)J.P * nmp;
     const double Ul = J.Up[l];
     // base row p = 0 (reading Q10), and the row flag of (l, v): it is reset
     // here and OR-ed by the step kernel for p >= 1
-    {
+    if (row_ok) {
         const double U1l = __dsub_rn(Ul, J.Up[0]);
         int64_t d;
         (void)transition(J, 1, l, v, U1l, &d);
         const bool ok = U1l <= J.tau && d <= (int64_t)(J.n_m - 1);
         double *o = J.table + (size_t)l * J.n_v * rowlen + (size_t)v * rowlen;
-        for (int m = lane; m < nmp; m += 32)
+        for (int m = hl; m < nmp; m += 16)
             o[m] = (m < J.n_m && U1l <= J.tau && (int64_t)m + d <= (int64_t)(J.n_m - 1)) ? U1l : MP_INF;
-        if (lane == 0) J.rowflag[(size_t)l * J.n_v + v] = ok ? 1u : 0u;
+        if (hl == 0) J.rowflag[(size_t)l * J.n_v + v] = ok ? 1u : 0u;
     }
     const int kmin = J.kwin[l];   // max(kmin_tau(l), kmin_W(l)), precomputed by window_kernel
     unsigned live = 0, useful = 0;
     int n = 0;
-    TransEntry *list = J.tlist + (size_t)v * J.code_cap;
-    for (int kb = kmin; kb <= l; kb += 32) {
-        const int k = kb + lane;
+    TransEntry *list = J.tlist + (size_t)(row_ok ? v : 0) * J.code_cap;
+    for (int kb = kmin; kb <= l; kb += 16) {   // same trip count in both halves (same job, layer)
+        const int k = kb + hl;
         int32_t tr = -1;
         double Ukl = 0.0;
         bool use = false;
-        if (k <= l) {
+        if (row_ok && k <= l) {
             Ukl = __dsub_rn(Ul, J.Up[k - 1]);
             tr = transition(J, k, l, v, Ukl, nullptr);
             if (tr >= 0) {
@@ -309,15 +312,15 @@ __global__ void __launch_bounds__(256, 4) trans_kernel(const Job *jobs, int l, i
                 useful += use;
             }
         }
-        const unsigned bal = __ballot_sync(0xffffffffu, use);
+        const unsigned bal = (__ballot_sync(0xffffffffu, use) >> (half * 16)) & 0xFFFFu;
         if (use) {
             TransEntry e;
             e.U = Ukl; e.code = tr; e.k = k;
-            list[n + __popc(bal & ((1u << lane) - 1u))] = e;
+            list[n + __popc(bal & ((1u << hl) - 1u))] = e;
         }
         n += __popc(bal);
     }
-    if (lane == 0) J.tcount[v] = n;
+    if (row_ok && hl == 0) J.tcount[v] = n;
     for (int o = 16; o > 0; o >>= 1) {
         live += __shfl_xor_sync(0xffffffffu, live, o);
         useful += __shfl_xor_sync(0xffffffffu, useful, o);
@@ -346,7 +349,7 @@ void launch_window(const Job *jobs, int n_jobs, int max_L, cudaStream_t s) {
 }
 
 void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, cudaStream_t s) {
-    trans_kernel<<<dim3((n_v_max + 7) / 8, n_jobs), 256, 0, s>>>(jobs, l, nmp);
+    trans_kernel<<<dim3((n_v_max + 15) / 16, n_jobs), 256, 0, s>>>(jobs, l, nmp);
 }
 
 // ---------------------------------------------------------------------------
