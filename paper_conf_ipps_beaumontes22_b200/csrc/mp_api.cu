@@ -46,6 +46,8 @@ struct madpipe_ctx {
     DevBuf tables, jobs, tiles, chains, chain_data, jl, counts, roots, trace, stages, scratch, codes, flags,
         tlist;
     cudaEvent_t ev_a = nullptr, ev_b = nullptr;
+    cudaStream_t aux = nullptr;        // second stream: trans_kernel(l+1) overlaps step(l)
+    cudaEvent_t ev_tr[4] = {}, ev_st[4] = {}, ev_w = nullptr;
     double sweep_ms = 0.0, step_ms = 0.0;
     int64_t launches = 0;
     int64_t h2d_bytes = 0, d2h_bytes = 0;
@@ -231,6 +233,12 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stre
     if (const char *e = getenv("MADPIPE_TILE_BLOCK")) c->tile_block = std::max(1, atoi(e));
     cudaEventCreate(&c->ev_a);
     cudaEventCreate(&c->ev_b);
+    cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking);
+    for (int i = 0; i < 4; i++) {
+        cudaEventCreateWithFlags(&c->ev_tr[i], cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&c->ev_st[i], cudaEventDisableTiming);
+    }
+    cudaEventCreateWithFlags(&c->ev_w, cudaEventDisableTiming);
     *out = c;
     return MADPIPE_OK;
 }
@@ -244,6 +252,12 @@ extern "C" void madpipe_ctx_destroy(madpipe_ctx *c) {
                       &c->counts, &c->roots, &c->trace, &c->stages, &c->scratch, &c->codes, &c->flags, &c->tlist};
     for (DevBuf *b : bufs) b->release();
     for (cudaEvent_t ev : c->ev_pool) cudaEventDestroy(ev);
+    if (c->aux) { cudaStreamSynchronize(c->aux); cudaStreamDestroy(c->aux); }
+    for (int i = 0; i < 4; i++) {
+        if (c->ev_tr[i]) cudaEventDestroy(c->ev_tr[i]);
+        if (c->ev_st[i]) cudaEventDestroy(c->ev_st[i]);
+    }
+    if (c->ev_w) cudaEventDestroy(c->ev_w);
     if (c->ev_a) cudaEventDestroy(c->ev_a);
     if (c->ev_b) cudaEventDestroy(c->ev_b);
     if (c->own_stream) cudaStreamDestroy(c->stream);
@@ -450,6 +464,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             hjobs[i].kmin_l = (int32_t *)((unsigned long long *)ctx->counts.p + 3 * nj) + i;
         }
         int n_v_max = 0;
+        size_t list_buf_entries = 0;
         if (ctx->kernel == 2) {
             // useful-transition lists of one layer: [job][v][maxL] entries + [job][v] counts
             size_t total = 0, vtotal = 0;
@@ -458,8 +473,10 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 vtotal += (size_t)J.n_v;
                 n_v_max = std::max(n_v_max, J.n_v);
             }
-            CUDA_TRY(ctx, ctx->tlist.ensure(total * sizeof(TransEntry)));
-            CUDA_TRY(ctx, ctx->codes.ensure(vtotal * sizeof(int32_t)));
+            // two buffers (layers l and l+1 are live at once when trans(l+1) overlaps step(l))
+            CUDA_TRY(ctx, ctx->tlist.ensure(2 * total * sizeof(TransEntry)));
+            CUDA_TRY(ctx, ctx->codes.ensure(2 * vtotal * sizeof(int32_t)));
+            list_buf_entries = total;
             size_t off = 0, voff = 0, ftotal = 0;
             for (auto &J : hjobs) {
                 J.tlist = (TransEntry *)ctx->tlist.p + off;
@@ -513,23 +530,32 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         if (ctx->kernel == 2) {
             launch_window(djobs, nj, maxL, ctx->stream);
             ctx->launches++;
+            CUDA_TRY(ctx, cudaEventRecord(ctx->ev_w, ctx->stream));
+            CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_w, 0));
         }
         for (int l = 1; l <= maxL; l++) {
+            const size_t buf_off = (size_t)(l & 1) * list_buf_entries;
             if (ctx->kernel == 2) {
-                launch_trans(djobs, nj, n_v_max, l, nmp, ctx->stream);
+                // trans(l) on the aux stream, overlapping step(l-1): it needs step(l-2) done
+                // (the flags of slabs <= l-2 and the list buffer l%2 it overwrites)
+                if (l >= 3) CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_st[(l - 2) & 3], 0));
+                launch_trans(djobs, nj, n_v_max, l, nmp, buf_off, /*verify_last=*/0, ctx->aux);
                 ctx->launches++;
+                CUDA_TRY(ctx, cudaEventRecord(ctx->ev_tr[l & 3], ctx->aux));
+                CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->stream, ctx->ev_tr[l & 3], 0));
             }
             // per-launch events bracket the step kernel alone (bench roofline)
             if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1)], ctx->stream);
             if (ctx->kernel == 2)
                 launch_step_persist(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, p_np, p_vb, nsg,
                                     persist_grid, (unsigned long long *)(ctx->prof ? ctx->profbuf.p : nullptr),
-                                    ctx->n_prod, ctx->tile_block, ctx->stream);
+                                    ctx->n_prod, ctx->tile_block, buf_off, ctx->stream);
             else if (ctx->kernel == 1)
                 launch_step_tma(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, smem_tma, ctx->stream);
             else
                 launch_step(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, ctx->stream);
             if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1) + 1], ctx->stream);
+            if (ctx->kernel == 2) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[l & 3], ctx->stream));
         }
         ctx->launches += maxL;
         launch_root(djobs, nj, nmp, jl_dev, roots_dev, taus_dev, ctx->stream);

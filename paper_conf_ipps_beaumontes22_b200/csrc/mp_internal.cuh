@@ -91,12 +91,13 @@ void launch_step_tma(const Job *jobs, const int32_t *tile_job, int n_tiles, int 
 int tma_smem_bytes(int vb, int np, int nmp);
 void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np,
                          int vb, int nsg, int grid, unsigned long long *prof, int n_prod, int tile_block,
-                         cudaStream_t s);
+                         size_t buf_off, cudaStream_t s);
 int persist_blocks_per_sm(int nmp, int np, int vb, int nsg, int n_prod);
 void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
 int persist_nsg(int np, int vb, int nmp);
 void tma_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
-void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, cudaStream_t s);
+void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int verify_last,
+                  cudaStream_t s);
 void launch_window(const Job *jobs, int n_jobs, int max_L, cudaStream_t s);
 void launch_lit_init(const Job *job, int n_t, double dt, int nmp, int64_t cells, cudaStream_t s);
 void launch_lit_step(const Job *job, int n_t, double dt, int nmp, int n_v, int P, int l, cudaStream_t s);

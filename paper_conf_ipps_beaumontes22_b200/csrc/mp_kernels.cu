@@ -263,10 +263,15 @@ void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, i
 // (a row that is +inf everywhere can only contribute +inf).  Also counts the
 // job's effective and useful relaxations.
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(256, 4) trans_kernel(const Job *jobs, int l, int nmp) {
-    // one half-warp per delay row v of the job (16 rows per CTA: the windows are
-    // short, and the kernel is latency-bound, so fewer, fuller warps win); the job
-    // descriptor is read once into shared memory
+__global__ void __launch_bounds__(64) trans_kernel(const Job *jobs, int l, int nmp, size_t buf_off,
+                                                   int verify_last) {
+    // one half-warp per delay row v of the job (4 rows per 64-thread CTA: small
+    // CTAs so that one fits on an SM beside the two resident step-kernel CTAs -- this
+    // kernel runs on a second stream, overlapped with the step kernel of layer l-1);
+    // the job descriptor is read once into shared memory.  buf_off selects the list
+    // buffer of layer l (double-buffered).  verify_last = 0: the source row of k = l
+    // (slab l-1) may still be being written by the concurrent step kernel, so its
+    // flag is not consulted -- that entry is kept (and counted as read).
     __shared__ Job sJ;
     if (threadIdx.x < sizeof(Job) / 8)
         reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
@@ -276,7 +281,7 @@ __global__ void __launch_bounds__(256, 4) trans_kernel(const Job *jobs, int l, i
     if (l > J.L) return;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int half = lane >> 4, hl = lane & 15;
-    const int v = blockIdx.x * 16 + warp * 2 + half;
+    const int v = blockIdx.x * 4 + warp * 2 + half;
     const bool row_ok = v < J.n_v;
     if (__ballot_sync(0xffffffffu, row_ok) == 0u) return;
     const size_t rowlen = (size_t)J.P * nmp;
@@ -296,7 +301,7 @@ __global__ void __launch_bounds__(256, 4) trans_kernel(const Job *jobs, int l, i
     const int kmin = J.kwin[l];   // max(kmin_tau(l), kmin_W(l)), precomputed by window_kernel
     unsigned live = 0, useful = 0;
     int n = 0;
-    TransEntry *list = J.tlist + (size_t)(row_ok ? v : 0) * J.code_cap;
+    TransEntry *list = J.tlist + buf_off + (size_t)(row_ok ? v : 0) * J.code_cap;
     for (int kb = kmin; kb <= l; kb += 16) {   // same trip count in both halves (same job, layer)
         const int k = kb + hl;
         int32_t tr = -1;
@@ -308,7 +313,7 @@ __global__ void __launch_bounds__(256, 4) trans_kernel(const Job *jobs, int l, i
             if (tr >= 0) {
                 live++;
                 // a source row that is +inf everywhere can only contribute +inf (exact skip)
-                use = J.rowflag[(size_t)(k - 1) * J.n_v + (tr & 0xFFFF)] != 0u;
+                use = (k == l && !verify_last) || J.rowflag[(size_t)(k - 1) * J.n_v + (tr & 0xFFFF)] != 0u;
                 useful += use;
             }
         }
@@ -320,7 +325,7 @@ __global__ void __launch_bounds__(256, 4) trans_kernel(const Job *jobs, int l, i
         }
         n += __popc(bal);
     }
-    if (row_ok && hl == 0) J.tcount[v] = n;
+    if (row_ok && hl == 0) J.tcount[buf_off / J.code_cap + v] = n;
     for (int o = 16; o > 0; o >>= 1) {
         live += __shfl_xor_sync(0xffffffffu, live, o);
         useful += __shfl_xor_sync(0xffffffffu, useful, o);
@@ -348,8 +353,9 @@ void launch_window(const Job *jobs, int n_jobs, int max_L, cudaStream_t s) {
     window_kernel<<<(n + 255) / 256, 256, 0, s>>>(jobs, n_jobs, max_L);
 }
 
-void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, cudaStream_t s) {
-    trans_kernel<<<dim3((n_v_max + 15) / 16, n_jobs), 256, 0, s>>>(jobs, l, nmp);
+void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int verify_last,
+                  cudaStream_t s) {
+    trans_kernel<<<dim3((n_v_max + 3) / 4, n_jobs), 64, 0, s>>>(jobs, l, nmp, buf_off, verify_last);
 }
 
 // ---------------------------------------------------------------------------

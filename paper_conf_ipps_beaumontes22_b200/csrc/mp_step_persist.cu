@@ -93,7 +93,7 @@ __global__ void __launch_bounds__(kPCons + 32 * kProdMax, 2) step_persist_kernel
                                                                       const int32_t *__restrict__ tile_job,
                                                                       int n_tiles, int l, int np_max, int vb,
                                                                       int nsg, unsigned long long *prof,
-                                                                      int n_prod, int tile_block) {
+                                                                      int n_prod, int tile_block, size_t buf_off) {
     // prof (optional, MADPIPE_PROF=1): cycle counters [0] producer total, [1] tile setup,
     // [2] list building, [3] issue, [4] producer waits on empty, [5] consumer total,
     // [6] consumer waits on full, [7] tiles
@@ -168,8 +168,9 @@ __global__ void __launch_bounds__(kPCons + 32 * kProdMax, 2) step_persist_kernel
             double *out = J.table + (size_t)l * slab;
             const bool my_ring = ir < my_rings && iw < vcount;
             // number of useful transitions of my ring's row (trans_kernel)
-            const int n_w = my_ring ? __ldg(J.tcount + v0 + iw) : 0;
-            const TransEntry *list = J.tlist + (size_t)(v0 + (my_ring ? iw : 0)) * J.code_cap;
+            // list buffer of layer l: buf_off entries (and buf_off / code_cap counts) in
+            const int n_w = my_ring ? __ldg(J.tcount + buf_off / J.code_cap + v0 + iw) : 0;
+            const TransEntry *list = J.tlist + buf_off + (size_t)(v0 + (my_ring ? iw : 0)) * J.code_cap;
             const int n_eff = my_ring ? (n_w > 0 ? n_w : 1) : 0;   // 1 = closing stage without data
             int max_n = n_eff;
             for (int o = 16; o > 0; o >>= 1) max_n = max(max_n, __shfl_xor_sync(0xffffffffu, max_n, o));
@@ -397,13 +398,13 @@ int persist_nsg(int np, int vb, int nmp) {
 
 void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np,
                          int vb, int nsg, int grid, unsigned long long *prof, int n_prod, int tile_block,
-                         cudaStream_t s) {
+                         size_t buf_off, cudaStream_t s) {
     const int smem = vb * nsg * (np + 1) * nmp * 8;
     switch (nmp) {
 #define MP_CASE(N)                                                                                      \
     case N:                                                                                             \
         cudaFuncSetAttribute(step_persist_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
-        step_persist_kernel<N><<<grid, kPCons + 32 * n_prod, smem, s>>>(jobs, tile_job, n_tiles, l, np, vb, nsg, prof, n_prod, tile_block); \
+        step_persist_kernel<N><<<grid, kPCons + 32 * n_prod, smem, s>>>(jobs, tile_job, n_tiles, l, np, vb, nsg, prof, n_prod, tile_block, buf_off); \
         break;
         MP_CASE(2) MP_CASE(4) MP_CASE(8) MP_CASE(16) MP_CASE(32) MP_CASE(64)
 #undef MP_CASE
