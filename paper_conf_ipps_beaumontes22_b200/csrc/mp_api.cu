@@ -53,7 +53,8 @@ struct madpipe_ctx {
     int64_t h2d_bytes = 0, d2h_bytes = 0;
     int64_t last_cell_updates = 0, last_effective = 0, last_useful = 0;
     int per_launch_timing = 0;
-    int kernel = 2;           // MADPIPE_KERNEL: v1 = plain loads, tma = per-tile TMA, persist (default)
+    int kernel = -1;          // MADPIPE_KERNEL: v1 = plain loads, tma = per-tile TMA, persist;
+                              // -1 (default): persist when a row segment is >= 1 KB, else v1
     int prof = 0;             // MADPIPE_PROF=1: cycle counters of the persistent step kernel to stderr
     int n_prod = 4;           // MADPIPE_NPROD: producer warps of the persistent step kernel (1..4)
     int tile_block = 1;       // MADPIPE_TILE_BLOCK: consecutive tiles per interleaved block (1 = round-robin)
@@ -226,6 +227,7 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stre
     const char *kern = getenv("MADPIPE_KERNEL");
     if (kern && strcmp(kern, "v1") == 0) c->kernel = 0;
     if (kern && strcmp(kern, "tma") == 0) c->kernel = 1;
+    if (kern && strcmp(kern, "persist") == 0) c->kernel = 2;
     cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device);
     const char *pf = getenv("MADPIPE_PROF");
     c->prof = pf && pf[0] == '1';
@@ -410,6 +412,15 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
     while (next < js.size()) {
         // ---- form a batch
         hjobs.clear(); htiles.clear(); ids.clear();
+        // step kernel of this batch (measured): the persistent TMA kernel moves
+        // one row segment per stage, which pays off from ~1 KB segments; below, plain loads win
+        int kern = ctx->kernel;
+        while (next < js.size() && early_exit && jl_host[js[next].chain] < js[next].j) next++;
+        if (kern < 0 && next < js.size()) {
+            int vb_, np_, npt_, nt_;
+            persist_geom(cs[js[next].chain].P, disc->n_delay, nmp, &vb_, &np_, &npt_, &nt_);
+            kern = (np_ + 1) * nmp * 8 >= 1024 ? 2 : 0;
+        }
         size_t used = 0;
         int maxL = 0;
         size_t max_slab = 0;
@@ -420,8 +431,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             const ChainSpec &c = cs[s.chain];
             const size_t bytes = table_doubles(c, disc) * 8;
             if (!hjobs.empty() && (used + bytes > budget || hjobs.size() >= cap_jobs)) break;
-            // the persistent step kernel needs one tile geometry per launch: uniform P
-            if (ctx->kernel == 2 && !hjobs.empty() && c.P != hjobs[0].P) break;
+            // one tile geometry (and one step kernel) per launch: uniform P
+            if (!hjobs.empty() && c.P != hjobs[0].P) break;
             if (hjobs.empty() && bytes > budget && bytes > ctx->tables.n) {
                 // a single job larger than the budget: try anyway (may fail with ENOMEM)
             }
@@ -434,9 +445,9 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             J.chain = s.chain;
             J.gid = (int32_t)next;
             int n_tiles;
-            if (ctx->kernel == 2) {
+            if (kern == 2) {
                 persist_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
-            } else if (ctx->kernel == 1) {
+            } else if (kern == 1) {
                 tma_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
                 smem_tma = std::max(smem_tma, tma_smem_bytes(J.vb, J.np, nmp));
             } else {
@@ -465,7 +476,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         }
         int n_v_max = 0;
         size_t list_buf_entries = 0;
-        if (ctx->kernel == 2) {
+        if (kern == 2) {
             // useful-transition lists of one layer: [job][v][maxL] entries + [job][v] counts
             size_t total = 0, vtotal = 0;
             for (auto &J : hjobs) {
@@ -508,7 +519,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         ctx->launches += 2;
         const int n_tiles = (int)htiles.size();
         int persist_grid = 0, nsg = 0, p_np = 0, p_vb = 0;
-        if (ctx->kernel == 2) {
+        if (kern == 2) {
             p_np = hjobs[0].np;
             p_vb = hjobs[0].vb;
             nsg = persist_nsg(p_np, p_vb, nmp);
@@ -527,7 +538,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 ctx->ev_pool.push_back(ev);
             }
         }
-        if (ctx->kernel == 2) {
+        if (kern == 2) {
             launch_window(djobs, nj, maxL, ctx->stream);
             ctx->launches++;
             CUDA_TRY(ctx, cudaEventRecord(ctx->ev_w, ctx->stream));
@@ -535,7 +546,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         }
         for (int l = 1; l <= maxL; l++) {
             const size_t buf_off = (size_t)(l & 1) * list_buf_entries;
-            if (ctx->kernel == 2) {
+            if (kern == 2) {
                 // trans(l) on the aux stream, overlapping step(l-1): it needs step(l-2) done
                 // (the flags of slabs <= l-2 and the list buffer l%2 it overwrites)
                 if (l >= 3) CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_st[(l - 2) & 3], 0));
@@ -546,16 +557,16 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             }
             // per-launch events bracket the step kernel alone (bench roofline)
             if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1)], ctx->stream);
-            if (ctx->kernel == 2)
+            if (kern == 2)
                 launch_step_persist(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, p_np, p_vb, nsg,
                                     persist_grid, (unsigned long long *)(ctx->prof ? ctx->profbuf.p : nullptr),
                                     ctx->n_prod, ctx->tile_block, buf_off, ctx->stream);
-            else if (ctx->kernel == 1)
+            else if (kern == 1)
                 launch_step_tma(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, smem_tma, ctx->stream);
             else
                 launch_step(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, ctx->stream);
             if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1) + 1], ctx->stream);
-            if (ctx->kernel == 2) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[l & 3], ctx->stream));
+            if (kern == 2) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[l & 3], ctx->stream));
         }
         ctx->launches += maxL;
         launch_root(djobs, nj, nmp, jl_dev, roots_dev, taus_dev, ctx->stream);

@@ -25,6 +25,27 @@ def ctx():
     c.close()
 
 
+def _ctx_with_kernel(kernel):
+    """A context whose step kernel is forced (MADPIPE_KERNEL is read at creation)."""
+    import os
+    old = os.environ.get("MADPIPE_KERNEL")
+    os.environ["MADPIPE_KERNEL"] = kernel
+    try:
+        return mp.Context(0)
+    finally:
+        if old is None:
+            del os.environ["MADPIPE_KERNEL"]
+        else:
+            os.environ["MADPIPE_KERNEL"] = old
+
+
+@pytest.fixture(scope="module", params=["persist", "v1", "tma"])
+def kctx(request):
+    c = _ctx_with_kernel(request.param)
+    yield c
+    c.close()
+
+
 def _args(cfg):
     return (cfg["P"], cfg["M"], cfg["beta"], cfg["n_mem"], cfg["n_delay"], cfg["n_periods"])
 
@@ -43,7 +64,8 @@ def _verify(ch, P, M, beta, res):
 
 
 # ---------------------------------------------------------------- toy: everything, every candidate
-def test_toy_full_tables_every_candidate(ctx):
+def test_toy_full_tables_every_candidate(kctx):
+    ctx = kctx
     cfg = configs.load("toy")
     ch = chaingen.make(cfg["chain"])
     a = _args(cfg)
@@ -79,7 +101,8 @@ def _fuzz_cases(n, seed):
         yield ch, P, M, beta, n_m, n_v, n_c, vr
 
 
-def test_fuzz_roots_tables_solutions(ctx):
+def test_fuzz_roots_tables_solutions(kctx):
+    ctx = kctx
     for ch, P, M, beta, n_m, n_v, n_c, vr in _fuzz_cases(120, 7):
         ref = oracle.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
         tau, root = ctx.candidates(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
