@@ -234,3 +234,28 @@ def test_coarse_to_fine_matches_full_sweep_when_monotone(ctx):
         ctf = ctx.solve(ch, *_args(cfg), early_exit=2)
         _same_solution(ctf, full)
         assert ctf["cell_updates"] <= full["cell_updates"] * 2
+
+
+@pytest.mark.parametrize("P,n_m,n_v,L", [(300, 4, 6, 9),      # ROW mode, 2 processor tiles
+                                         (40, 33, 5, 8),      # PAIR mode (NMP 64), 5 processor tiles
+                                         (20, 17, 4, 10),     # PAIR mode (NMP 32), 2 processor tiles
+                                         (5, 8, 300, 12),     # delay levels above 255
+                                         (1, 8, 16, 30),      # P = 1: base rows only
+                                         (3, 2, 2, 1)])       # L = 1, smallest grids
+def test_geometry_extremes(P, n_m, n_v, L):
+    """Tile geometries the configs do not reach (processor tiling, wide delay grids,
+    P = 1, L = 1), for every step kernel, against the oracle."""
+    rng = np.random.default_rng(P * 1000 + n_m)
+    ch = chaingen.tiny(rng, L)
+    M = int((3 * ch["W"].sum() + 3 * ch["a"].sum()) * 0.6) + 1
+    n_c = 9
+    ref = oracle.solve(ch, P, M, 25.0, n_m, n_v, n_c, v_range=1, n_threads=4)
+    for kernel in ("persist", "v1", "tma"):
+        c = _ctx_with_kernel(kernel)
+        try:
+            tau, root = c.candidates(ch, P, M, 25.0, n_m, n_v, n_c, v_range=1)
+            assert np.array_equal(root, ref["root"]), kernel
+            got = c.solve(ch, P, M, 25.0, n_m, n_v, n_c, v_range=1)
+            _same_solution(got, ref)
+        finally:
+            c.close()
