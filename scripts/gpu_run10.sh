@@ -1,0 +1,5 @@
+cd $GRAFT_REPO_ROOT
+python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?" >> gpurun_out/smoke.log
+timeout 1800 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_gpu.log 2>&1
+timeout 900 python bench.py --config gpt --steps 3 --warmup 3 > gpurun_out/bench_gpt.json 2> gpurun_out/bench_gpt.err
+echo done
