@@ -108,7 +108,7 @@ const char *madpipe_last_error(const madpipe_ctx *ctx);   /* ctx may be NULL */
 
 /* ---- host-only helpers (no GPU needed) ------------------------------------ */
 /* Check every argument rule of this header; MADPIPE_OK or MADPIPE_EINVAL.
- * Rules: 1 <= L <= 65535; 1 <= P <= 65535; M > 0; beta > 0 and not NaN (beta = +inf allowed:
+ * Rules: L >= 1; P >= 1; M > 0; beta > 0 and not NaN (beta = +inf allowed:
  * C = 0); uF, uB finite, >= 0, uF+uB > 0; W >= 0; a >= 0; 2 <= n_mem <= 64;
  * 2 <= n_delay <= 65535; n_periods >= 1; v_range in {0,1}; int64 overflow
  * guards 3*sum W + (g_max)*sum a and (M-1) + (n_mem-1)*(3 sum W + g_max sum a). */

@@ -115,8 +115,8 @@ static int validate_impl(const madpipe_chain *ch, int32_t P, int64_t M, double b
                          const madpipe_disc *disc, bool host_arrays, std::string *why) {
     auto bad = [&](const char *msg) { if (why) *why = msg; return MADPIPE_EINVAL; };
     if (!ch || !disc) return bad("null chain or disc");
-    if (ch->L < 1 || ch->L > 65535) return bad("L outside [1, 65535]");
-    if (P < 1 || P > 65535) return bad("P outside [1, 65535]");
+    if (ch->L < 1) return bad("L < 1");
+    if (P < 1) return bad("P < 1");
     if (M <= 0) return bad("M <= 0");
     if (!(beta > 0.0)) return bad("beta must be > 0 (and not NaN)");
     if (disc->n_mem < 2 || disc->n_mem > 64) return bad("n_mem outside [2, 64]");

@@ -46,8 +46,7 @@ struct Job {
     int32_t *kmin_l;    // window start of layer l for this job (written by trans_kernel)
     int32_t code_cap;   // row capacity of codes (>= longest window of the batch)
     int32_t pad_;
-    uint32_t *rowflag;  // [(L+1)][n_v]: p_first of row (l, v): smallest p holding a finite value, P if
-                        // none (A is non-increasing in p; persist path)
+    uint32_t *rowflag;  // [(L+1)][n_v]: 1 if row (l, v) holds a finite value (persist path)
     unsigned long long *useful;  // live relaxations whose source row is not all +inf
     struct TransEntry *tlist;    // [n_v][code_cap] useful transitions of layer l (persist path)
     int32_t *tcount;             // [n_v] their number
@@ -58,8 +57,7 @@ struct Job {
 struct TransEntry {
     double U;        // U(k,l)
     int32_t code;    // pack_trans(v', d, nf)
-    uint16_t k;
-    uint16_t ps;     // p_first of the source row A[k-1][v'] (0 if not verified)
+    int32_t k;
 };
 
 // Result of a traceback, written by traceback_kernel.

@@ -104,9 +104,9 @@ void launch_jobs_init(Job *jobs, int n_jobs, cudaStream_t s) {
 __global__ void init_slab0_kernel(const Job *jobs, int nmp) {
     const Job &J = jobs[blockIdx.y];
     const int64_t cells = (int64_t)J.n_v * J.P * nmp;
-    if (J.rowflag)   // slab 0 is 0 everywhere: p_first = 0
+    if (J.rowflag)
         for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < J.n_v; v += gridDim.x * blockDim.x)
-            J.rowflag[v] = 0u;
+            J.rowflag[v] = 1u;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cells;
          i += (int64_t)gridDim.x * blockDim.x) {
         const int m = (int)(i % nmp);
@@ -296,11 +296,10 @@ __global__ void __launch_bounds__(64) trans_kernel(const Job *jobs, int l, int n
         double *o = J.table + (size_t)l * J.n_v * rowlen + (size_t)v * rowlen;
         for (int m = hl; m < nmp; m += 16)
             o[m] = (m < J.n_m && U1l <= J.tau && (int64_t)m + d <= (int64_t)(J.n_m - 1)) ? U1l : MP_INF;
-        if (hl == 0) J.rowflag[(size_t)l * J.n_v + v] = ok ? 0u : (uint32_t)J.P;   // p_first (min-ed by the step)
+        if (hl == 0) J.rowflag[(size_t)l * J.n_v + v] = ok ? 1u : 0u;
     }
     const int kmin = J.kwin[l];   // max(kmin_tau(l), kmin_W(l)), precomputed by window_kernel
-    unsigned live = 0;
-    unsigned long long useful = 0;   // relaxations with a finite source candidate
+    unsigned live = 0, useful = 0;
     int n = 0;
     TransEntry *list = J.tlist + buf_off + (size_t)(row_ok ? v : 0) * J.code_cap;
     for (int kb = kmin; kb <= l; kb += 16) {   // same trip count in both halves (same job, layer)
@@ -308,23 +307,20 @@ __global__ void __launch_bounds__(64) trans_kernel(const Job *jobs, int l, int n
         int32_t tr = -1;
         double Ukl = 0.0;
         bool use = false;
-        uint32_t ps = 0;
         if (row_ok && k <= l) {
             Ukl = __dsub_rn(Ul, J.Up[k - 1]);
             tr = transition(J, k, l, v, Ukl, nullptr);
             if (tr >= 0) {
                 live++;
-                // the source row's finite cells are {p >= ps}; a row that is +inf
-                // everywhere (ps = P) can only contribute +inf (exact skip)
-                if (!(k == l && !verify_last)) ps = J.rowflag[(size_t)(k - 1) * J.n_v + (tr & 0xFFFF)];
-                use = ps < (uint32_t)J.P;
-                if (use) useful += (unsigned long long)(J.P - max(1, (int)ps));
+                // a source row that is +inf everywhere can only contribute +inf (exact skip)
+                use = (k == l && !verify_last) || J.rowflag[(size_t)(k - 1) * J.n_v + (tr & 0xFFFF)] != 0u;
+                useful += use;
             }
         }
         const unsigned bal = (__ballot_sync(0xffffffffu, use) >> (half * 16)) & 0xFFFFu;
         if (use) {
             TransEntry e;
-            e.U = Ukl; e.code = tr; e.k = (uint16_t)k; e.ps = (uint16_t)ps;
+            e.U = Ukl; e.code = tr; e.k = k;
             list[n + __popc(bal & ((1u << hl) - 1u))] = e;
         }
         n += __popc(bal);
@@ -337,7 +333,7 @@ __global__ void __launch_bounds__(64) trans_kernel(const Job *jobs, int l, int n
     if (lane == 0 && live && J.P > 1) {
         const unsigned long long per = (unsigned long long)(J.P - 1) * (unsigned long long)J.n_m;
         atomicAdd(J.eff, (unsigned long long)live * per);
-        if (useful) atomicAdd(J.useful, useful * (unsigned long long)J.n_m);
+        if (useful) atomicAdd(J.useful, (unsigned long long)useful * per);
     }
 }
 

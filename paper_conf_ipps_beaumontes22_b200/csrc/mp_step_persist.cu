@@ -84,9 +84,8 @@ struct SlotMeta {
     double U;           // U(k,l)
     int32_t tr;         // transition code
     int32_t np;         // processor rows of the tile (<= np_max)
-    int32_t pso;        // slot sub-row 0 holds source processor p_lo - 1 + pso (trimmed start)
-    int32_t p_lo;       // first output processor of the tile
     int16_t n_m, flags; // flags: 1 = last stage of the row, 2 = no data, 4 = terminate
+    int32_t pad_;
 };
 
 template <int NMP>
@@ -195,27 +194,20 @@ __global__ void __launch_bounds__(kPCons + 32 * kProdMax, 2) step_persist_kernel
                     M.flag = J.rowflag + (size_t)l * J.n_v + v0 + iw;
                     M.tau = J.tau;
                     M.np = np;
-                    M.p_lo = p_lo;
                     M.n_m = (int16_t)J.n_m;
-                    // copy only the source sub-rows that can be finite: processors
-                    // [max(p_lo-1, ps), p_lo+np-1] (A is non-increasing in p)
-                    const int pso = n_w > 0 ? max(0, (int)e.ps - (p_lo - 1)) : 0;
-                    if (n_w == 0 || pso > np) {
-                        M.flags = (int16_t)((n_w == 0 || q == n_w - 1 ? 1 : 0) | 2);
+                    if (n_w == 0) {
+                        M.flags = 1 | 2;
                         M.tr = -1;
-                        M.pso = 0;
                         mbar_arrive(full0 + 8 * slot);
                     } else {
-                        const uint32_t bytes = seg_bytes - (uint32_t)pso * NMP * 8u;
                         bulk_g2s(ring_s + 8u * (uint32_t)(slot * seg_doubles),
                                  J.table + (size_t)(e.k - 1) * slab + (size_t)(e.code & 0xFFFF) * rowlen +
-                                     (size_t)(p_lo - 1 + pso) * NMP,
-                                 bytes, full0 + 8 * slot);
+                                     (size_t)(p_lo - 1) * NMP,
+                                 seg_bytes, full0 + 8 * slot);
                         M.flags = (int16_t)(q == n_w - 1 ? 1 : 0);
                         M.tr = e.code;
                         M.U = e.U;
-                        M.pso = pso;
-                        mbar_arrive_expect_tx(full0 + 8 * slot, bytes);
+                        mbar_arrive_expect_tx(full0 + 8 * slot, seg_bytes);
                     }
                 }
                 __syncwarp();
@@ -287,15 +279,12 @@ __global__ void __launch_bounds__(kPCons + 32 * kProdMax, 2) step_persist_kernel
         const bool active = pp_off < np;
         if (!(flags & 2) && active) {
             const int32_t tr = M.tr;
-            // slot sub-row i holds source processor p_lo - 1 + pso + i
-            const int pso = M.pso;
-            const double *rowN = ring + (size_t)slot * seg_doubles + (pp_off - pso) * NMP;   // processor p-1
-            const double *rowS = rowN + NMP;                                                  // processor p
-            const bool hasN = pp_off >= pso, hasS = pp_off + 1 >= pso;
+            const double *rowN = ring + (size_t)slot * seg_doubles + pp_off * NMP;   // processor p-1
+            const double *rowS = rowN + NMP;                                          // processor p
             const int d = (tr >> 16) & 0xFF;
             const double U = M.U;
             if (ROW) {
-                if ((tr & (1 << 24)) && hasN) {                 // N
+                if (tr & (1 << 24)) {                           // N
 #pragma unroll
                     for (int c = 0; c < C; c++) {
                         const int j = (c + rot) & (C - 1);
@@ -304,7 +293,7 @@ __global__ void __launch_bounds__(kPCons + 32 * kProdMax, 2) step_persist_kernel
                         best[2 * c + 1] = dmin(best[2 * c + 1], x.y);
                     }
                 }
-                if (d <= n_m - 1 && hasS) {                     // S
+                if (d <= n_m - 1) {                             // S
                     if ((d & 1) == 0) {
                         const int e = d >> 1;
 #pragma unroll
@@ -329,13 +318,13 @@ __global__ void __launch_bounds__(kPCons + 32 * kProdMax, 2) step_persist_kernel
                     }
                 }
             } else {
-                if ((tr & (1 << 24)) && hasN) {
+                if (tr & (1 << 24)) {
                     const double2 x = *reinterpret_cast<const double2 *>(rowN + 2 * h);
                     best[0] = dmin(best[0], x.x);
                     best[1] = dmin(best[1], x.y);
                 }
                 const int m0 = 2 * h + d;
-                if (m0 <= n_m - 1 && hasS) {
+                if (m0 <= n_m - 1) {
                     double y0, y1;
                     if ((d & 1) == 0) {
                         const double2 y = *reinterpret_cast<const double2 *>(rowS + m0);
@@ -372,9 +361,7 @@ __global__ void __launch_bounds__(kPCons + 32 * kProdMax, 2) step_persist_kernel
                     *reinterpret_cast<double2 *>(o + 2 * h) = r;
                 }
             }
-            // p_first of the row: smallest processor with a finite value (A is non-increasing in p)
-            const int pf = __reduce_min_sync(0xffffffffu, fin ? (int)(M.p_lo + pp_off) : 0x7fffffff);
-            if (lane == 0 && pf != 0x7fffffff) atomicMin(M.flag, (uint32_t)pf);
+            if (__ballot_sync(0xffffffffu, fin) && lane == 0) atomicOr(M.flag, 1u);
 #pragma unroll
             for (int i = 0; i < NB; i++) best[i] = MP_INF;
         }
