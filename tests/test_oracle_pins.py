@@ -339,3 +339,24 @@ def test_tie_break_smallest_split_first():
                         assert ARG[l, p, v, m] == (min(codes) if codes else -1)
                         n_ties += len(codes) > 1
     assert n_ties > 50
+
+
+def test_table_monotone_in_processors():
+    """Invariant (used by the kernels' sub-row trimming): with one more
+    normal GPU available every allocation stays possible (a GPU may stay unused,
+    T(0,p,..) = t_P for any p), so A[l][p] <= A[l][p-1] elementwise, and the
+    finite cells of a row (l, v) form an up-set {p >= p_first}."""
+    rng = np.random.default_rng(71)
+    for _ in range(40):
+        ch, P, M, beta, n_m, n_v, vr = _rand_case(rng, L=int(rng.integers(3, 10)), P=int(rng.integers(2, 7)))
+        pre = oracle.prep(ch, P, beta)
+        tau = pre["lb"] + rng.uniform(0.0, 1.0) * (pre["ub"] - pre["lb"])
+        A, _, _ = oracle.table(ch, P, M, beta, n_m, n_v, vr, tau, with_arg=False)
+        assert np.all(A[:, 1:] <= A[:, :-1])
+        fin = np.isfinite(A).any(axis=3)                       # [l][p][v]
+        for l in range(A.shape[0]):
+            for v in range(n_v):
+                col = fin[l, :, v]
+                if col.any():
+                    first = int(np.argmax(col))
+                    assert col[first:].all()
