@@ -189,6 +189,15 @@ int madpipe_last_io(const madpipe_ctx *ctx, int64_t *h2d_bytes, int64_t *d2h_byt
  * ones the default step kernel reads (0 for the other step kernels). */
 int madpipe_last_counts(const madpipe_ctx *ctx, int64_t *cell_updates, int64_t *effective_updates,
                         int64_t *useful_updates);
+/* Algorithmic bytes of the step kernel in the last sweep, the
+ * numerator of the bench's roofline: load_bytes = every source-row segment the
+ * step kernel brings on chip ((np+1) processor rows of the padded n_mem levels,
+ * fp64, per processor tile; the two-layer kernel loads a row shared by both of
+ * its layers once), store_bytes = every output row p >= 1 it writes.  segments =
+ * the number of merged source segments of the two-layer kernel (0 otherwise).
+ * Host-computed from the device counters; no GPU access. */
+int madpipe_last_step_bytes(const madpipe_ctx *ctx, int64_t *load_bytes, int64_t *store_bytes,
+                            int64_t *segments);
 
 /* ---- NEXT row f2: the 1F1B* pattern of a contiguous allocation (host only) --
  * For stages s_1..s_N (one per GPU, tiling layers 1..L in order; e.g. a

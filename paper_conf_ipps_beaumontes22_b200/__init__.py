@@ -232,6 +232,12 @@ class Context:
         N.check(self._lib.madpipe_last_counts(self.h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)))
         return dict(cell_updates=a.value, effective_updates=b.value, useful_updates=c.value)
 
+    def last_step_bytes(self):
+        """Algorithmic bytes of the step kernel in the last sweep (madpipe_last_step_bytes)."""
+        a = ctypes.c_int64(); b = ctypes.c_int64(); c = ctypes.c_int64()
+        N.check(self._lib.madpipe_last_step_bytes(self.h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)))
+        return dict(load_bytes=a.value, store_bytes=b.value, segments=c.value)
+
     def last_timing(self):
         s = ctypes.c_double(); k = ctypes.c_double(); n = ctypes.c_int64()
         N.check(self._lib.madpipe_last_timing(self.h, ctypes.byref(s), ctypes.byref(k), ctypes.byref(n)))

@@ -82,6 +82,7 @@ def lib():
         "madpipe_set_timing": (ctypes.c_int, [vp, ctypes.c_int]),
         "madpipe_last_io": (ctypes.c_int, [vp, _i64p, _i64p]),
         "madpipe_last_counts": (ctypes.c_int, [vp, _i64p, _i64p, _i64p]),
+        "madpipe_last_step_bytes": (ctypes.c_int, [vp, _i64p, _i64p, _i64p]),
         "madpipe_solve_paper": (ctypes.c_int, [vp, cp, ctypes.c_int32, ctypes.c_int64, ctypes.c_double,
                                                ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ap,
                                                _dp, _dp]),
@@ -103,7 +104,7 @@ EXPORTED = ["madpipe_ctx_create", "madpipe_ctx_destroy", "madpipe_last_error", "
             "madpipe_shard", "madpipe_cell_updates", "madpipe_solve", "madpipe_solve_dev",
             "madpipe_sweep", "madpipe_resolve", "madpipe_solve_batch", "madpipe_candidates",
             "madpipe_dp_table", "madpipe_last_timing", "madpipe_set_timing", "madpipe_last_io",
-            "madpipe_last_counts", "madpipe_schedule", "madpipe_solve_paper", "madpipe_literal_table"]
+            "madpipe_last_counts", "madpipe_last_step_bytes", "madpipe_schedule", "madpipe_solve_paper", "madpipe_literal_table"]
 
 
 class MadpipeError(RuntimeError):

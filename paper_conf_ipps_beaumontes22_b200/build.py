@@ -14,7 +14,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libmadpipe.so")
-SOURCES = ["mp_kernels.cu", "mp_step_tma.cu", "mp_step_persist.cu", "mp_api.cu", "mp_schedule.cu", "mp_literal.cu"]
+SOURCES = ["mp_kernels.cu", "mp_step_tma.cu", "mp_step_persist.cu", "mp_step_pair.cu", "mp_api.cu", "mp_schedule.cu", "mp_literal.cu"]
 HEADERS = ["mp_internal.cuh", "mp_device.cuh", os.path.join("..", "..", "include", "madpipe.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -51,7 +51,8 @@ struct madpipe_ctx {
     double sweep_ms = 0.0, step_ms = 0.0;
     int64_t launches = 0;
     int64_t h2d_bytes = 0, d2h_bytes = 0;
-    int64_t last_cell_updates = 0, last_effective = 0, last_useful = 0;
+    int64_t last_cell_updates = 0, last_effective = 0, last_useful = 0, last_segs = 0;
+    int64_t last_load_bytes = 0, last_store_bytes = 0;   // step kernel: source segments in, rows out
     int per_launch_timing = 0;
     int kernel = -1;          // MADPIPE_KERNEL: v1 = plain loads, tma = per-tile TMA, persist;
                               // -1 (default): persist when a row segment is >= 1 KB, else v1
@@ -60,6 +61,7 @@ struct madpipe_ctx {
     int tile_block = 1;       // MADPIPE_TILE_BLOCK: consecutive tiles per interleaved block (1 = round-robin)
     DevBuf profbuf;
     int num_sms = 148;
+    int n_rec = 0;            // step-kernel launches bracketed by per-launch events in the last batch
     std::vector<cudaEvent_t> ev_pool;
 };
 
@@ -228,6 +230,7 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stre
     if (kern && strcmp(kern, "v1") == 0) c->kernel = 0;
     if (kern && strcmp(kern, "tma") == 0) c->kernel = 1;
     if (kern && strcmp(kern, "persist") == 0) c->kernel = 2;
+    if (kern && strcmp(kern, "pair") == 0) c->kernel = 3;
     cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device);
     const char *pf = getenv("MADPIPE_PROF");
     c->prof = pf && pf[0] == '1';
@@ -281,6 +284,15 @@ extern "C" int madpipe_last_counts(const madpipe_ctx *c, int64_t *cell_updates,
     if (cell_updates) *cell_updates = c->last_cell_updates;
     if (effective_updates) *effective_updates = c->last_effective;
     if (useful_updates) *useful_updates = c->last_useful;
+    return MADPIPE_OK;
+}
+
+extern "C" int madpipe_last_step_bytes(const madpipe_ctx *c, int64_t *load_bytes, int64_t *store_bytes,
+                                       int64_t *segments) {
+    if (!c) return MADPIPE_EINVAL;
+    if (load_bytes) *load_bytes = c->last_load_bytes;
+    if (store_bytes) *store_bytes = c->last_store_bytes;
+    if (segments) *segments = c->last_segs;
     return MADPIPE_OK;
 }
 
@@ -399,7 +411,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
     size_t next = 0;
     if (timed) {
         ctx->sweep_ms = 0.0; ctx->step_ms = 0.0;
-        ctx->last_cell_updates = 0; ctx->last_effective = 0; ctx->last_useful = 0;
+        ctx->last_cell_updates = 0; ctx->last_effective = 0; ctx->last_useful = 0; ctx->last_segs = 0;
+        ctx->last_load_bytes = 0; ctx->last_store_bytes = 0;
     }
     std::vector<Job> hjobs;
     std::vector<int32_t> htiles;
@@ -416,6 +429,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         // one row segment per stage, which pays off from ~1 KB segments; below, plain loads win
         int kern = ctx->kernel;
         while (next < js.size() && early_exit && jl_host[js[next].chain] < js[next].j) next++;
+        if (kern == 3 && next < js.size() && !pair_supported(cs[js[next].chain].P, nmp)) kern = -1;
         if (kern < 0 && next < js.size()) {
             int vb_, np_, npt_, nt_;
             persist_geom(cs[js[next].chain].P, disc->n_delay, nmp, &vb_, &np_, &npt_, &nt_);
@@ -445,7 +459,11 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             J.chain = s.chain;
             J.gid = (int32_t)next;
             int n_tiles;
-            if (kern == 2) {
+            if (kern == 3) {
+                int nvt;
+                pair_geom(c.P, disc->n_delay, &J.np, &J.n_ptiles, &nvt, &n_tiles);
+                J.vb = 0;
+            } else if (kern == 2) {
                 persist_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
             } else if (kern == 1) {
                 tma_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
@@ -468,14 +486,52 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         const int nj = (int)hjobs.size();
         CUDA_TRY(ctx, ctx->jobs.ensure(sizeof(Job) * nj));
         CUDA_TRY(ctx, ctx->tiles.ensure(sizeof(int32_t) * htiles.size()));
-        CUDA_TRY(ctx, ctx->counts.ensure(sizeof(unsigned long long) * 3 * nj + sizeof(int32_t) * nj));
+        CUDA_TRY(ctx, ctx->counts.ensure(sizeof(unsigned long long) * 4 * nj + sizeof(int32_t) * nj));
         for (int i = 0; i < nj; i++) {
             hjobs[i].eff = (unsigned long long *)ctx->counts.p + nj + i;
             hjobs[i].useful = (unsigned long long *)ctx->counts.p + 2 * nj + i;
-            hjobs[i].kmin_l = (int32_t *)((unsigned long long *)ctx->counts.p + 3 * nj) + i;
+            hjobs[i].segs = (unsigned long long *)ctx->counts.p + 3 * nj + i;
+            hjobs[i].kmin_l = (int32_t *)((unsigned long long *)ctx->counts.p + 4 * nj) + i;
         }
         int n_v_max = 0;
-        size_t list_buf_entries = 0;
+        size_t list_buf_entries = 0, cnt_buf_entries = 0;
+        if (kern == 3) {
+            // merged two-layer lists: [job][v-tile][cap] PairEntry + [job][v-tile] counts, two buffers
+            const int cap = pair_list_cap(maxL);
+            size_t total = 0, vtotal = 0;
+            for (auto &J : hjobs) {
+                int np_, npt_, nvt_, nt_;
+                pair_geom(J.P, J.n_v, &np_, &npt_, &nvt_, &nt_);
+                total += (size_t)nvt_ * (size_t)cap;
+                vtotal += (size_t)nvt_;
+                n_v_max = std::max(n_v_max, J.n_v);
+            }
+            CUDA_TRY(ctx, ctx->tlist.ensure(2 * total * pair_entry_bytes()));
+            CUDA_TRY(ctx, ctx->codes.ensure(2 * vtotal * sizeof(int32_t)));
+            list_buf_entries = total;
+            cnt_buf_entries = vtotal;
+            size_t off = 0, voff = 0, ftotal = 0, wtotal = 0;
+            for (auto &J : hjobs) {
+                int np_, npt_, nvt_, nt_;
+                pair_geom(J.P, J.n_v, &np_, &npt_, &nvt_, &nt_);
+                J.tlist = (TransEntry *)((char *)ctx->tlist.p + off * pair_entry_bytes());
+                J.tcount = (int32_t *)ctx->codes.p + voff;
+                J.code_cap = cap;
+                off += (size_t)nvt_ * (size_t)cap;
+                voff += (size_t)nvt_;
+                ftotal += (size_t)(J.L + 1) * (size_t)J.n_v;
+                wtotal += (size_t)(J.L + 1);
+            }
+            CUDA_TRY(ctx, ctx->flags.ensure(ftotal * sizeof(uint32_t) + wtotal * sizeof(int32_t)));
+            size_t foff = 0, woff = 0;
+            int32_t *wbase = (int32_t *)((uint32_t *)ctx->flags.p + ftotal);
+            for (auto &J : hjobs) {
+                J.rowflag = (uint32_t *)ctx->flags.p + foff;
+                foff += (size_t)(J.L + 1) * (size_t)J.n_v;
+                J.kwin = wbase + woff;
+                woff += (size_t)(J.L + 1);
+            }
+        }
         if (kern == 2) {
             // useful-transition lists of one layer: [job][v][maxL] entries + [job][v] counts
             size_t total = 0, vtotal = 0;
@@ -512,13 +568,19 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         Job *djobs = (Job *)ctx->jobs.p;
         CUDA_TRY(ctx, h2d(ctx, djobs, hjobs.data(), sizeof(Job) * nj));
         CUDA_TRY(ctx, h2d(ctx, ctx->tiles.p, htiles.data(), sizeof(int32_t) * htiles.size()));
-        CUDA_TRY(ctx, cudaMemsetAsync(ctx->counts.p, 0, sizeof(unsigned long long) * 3 * nj, ctx->stream));
+        CUDA_TRY(ctx, cudaMemsetAsync(ctx->counts.p, 0, sizeof(unsigned long long) * 4 * nj, ctx->stream));
         if (timed) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_a, ctx->stream));
         launch_jobs_init(djobs, nj, ctx->stream);
         launch_init_slab0(djobs, nj, nmp, (int)std::min(max_slab, (size_t)INT32_MAX), ctx->stream);
         ctx->launches += 2;
         const int n_tiles = (int)htiles.size();
         int persist_grid = 0, nsg = 0, p_np = 0, p_vb = 0;
+        if (kern == 3) {
+            p_np = hjobs[0].np;
+            nsg = pair_nsl(p_np, nmp);
+            if (nsg < 4) return fail(ctx, MADPIPE_EINVAL, "row segment too large for the pair step kernel ring");
+            persist_grid = std::min(n_tiles, ctx->num_sms);
+        }
         if (kern == 2) {
             p_np = hjobs[0].np;
             p_vb = hjobs[0].vb;
@@ -538,6 +600,26 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 ctx->ev_pool.push_back(ev);
             }
         }
+        if (kern == 3) {
+            launch_window(djobs, nj, maxL, ctx->stream);
+            ctx->launches++;
+            int n_rec = 0;
+            for (int l = 1; l <= maxL; l += 2) {
+                const int b = (l >> 1) & 1;   // list buffer (double-buffered)
+                launch_pair_trans(djobs, nj, n_v_max, l, nmp, b * list_buf_entries, b * cnt_buf_entries, ctx->stream);
+                if (per_launch) cudaEventRecord(ctx->ev_pool[2 * n_rec], ctx->stream);
+                launch_pair_step(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, p_np, nsg, persist_grid,
+                                 b * list_buf_entries, b * cnt_buf_entries, ctx->stream);
+                if (per_launch) cudaEventRecord(ctx->ev_pool[2 * n_rec + 1], ctx->stream);
+                n_rec++;
+                ctx->launches += 2;
+                if (l + 1 <= maxL) {
+                    launch_pair_fixup(djobs, nj, n_v_max, l + 1, nmp, ctx->stream);
+                    ctx->launches++;
+                }
+            }
+            ctx->n_rec = n_rec;
+        } else {
         if (kern == 2) {
             launch_window(djobs, nj, maxL, ctx->stream);
             ctx->launches++;
@@ -569,6 +651,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             if (kern == 2) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[l & 3], ctx->stream));
         }
         ctx->launches += maxL;
+        ctx->n_rec = maxL;
+        }
         launch_root(djobs, nj, nmp, jl_dev, roots_dev, taus_dev, ctx->stream);
         launch_count(djobs, nj, (unsigned long long *)ctx->counts.p, ctx->stream);
         ctx->launches += 2;
@@ -589,8 +673,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             int rc = hook->after_batch(ctx, ids, djobs);
             if (rc) return rc;
         }
-        hcounts.resize(3 * nj);
-        CUDA_TRY(ctx, d2h(ctx, hcounts.data(), ctx->counts.p, sizeof(unsigned long long) * 3 * nj));
+        hcounts.resize(4 * nj);
+        CUDA_TRY(ctx, d2h(ctx, hcounts.data(), ctx->counts.p, sizeof(unsigned long long) * 4 * nj));
         if (early_exit)
             CUDA_TRY(ctx, d2h(ctx, jl_host.data(), jl_dev, sizeof(int32_t) * n_chains));
         CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
@@ -601,6 +685,17 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 ctx->last_cell_updates += (int64_t)hcounts[i];
                 ctx->last_effective += (int64_t)hcounts[nj + i];
                 ctx->last_useful += (int64_t)hcounts[2 * nj + i];
+                ctx->last_segs += (int64_t)hcounts[3 * nj + i];
+                // algorithmic bytes of the step kernel: every source
+                // segment it brings on chip -- (np+1) rows of nmp doubles per p-tile --
+                // and every output row p >= 1 it stores
+                const Job &J = hjobs[i];
+                const int64_t rowb = (int64_t)nmp * 8;
+                const int64_t seg = (int64_t)(J.P - 1 + J.n_ptiles) * rowb;
+                if (kern == 3) ctx->last_load_bytes += (int64_t)hcounts[3 * nj + i] * seg;
+                else if (kern == 2 && J.P > 1)
+                    ctx->last_load_bytes += (int64_t)(hcounts[2 * nj + i] / ((uint64_t)(J.P - 1) * J.n_m)) * seg;
+                ctx->last_store_bytes += (int64_t)J.L * J.n_v * (J.P - 1) * rowb;
             }
         }
         if (timed) {
@@ -608,7 +703,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b);
             ctx->sweep_ms += ms;
             if (per_launch) {
-                for (int l = 1; l <= maxL; l++) {
+                for (int l = 1; l <= ctx->n_rec; l++) {
                     float m2 = 0.f;
                     cudaEventElapsedTime(&m2, ctx->ev_pool[2 * (l - 1)], ctx->ev_pool[2 * (l - 1) + 1]);
                     ctx->step_ms += m2;

@@ -51,6 +51,7 @@ struct Job {
     struct TransEntry *tlist;    // [n_v][code_cap] useful transitions of layer l (persist path)
     int32_t *tcount;             // [n_v] their number
     int32_t *kwin;               // [L+1] window start max(kmin_tau(l), kmin_W(l)) (window_kernel)
+    unsigned long long *segs;    // source segments loaded (pair path: merged list entries)
 };
 
 // One useful transition of layer l for delay row v, in ascending k (trans_kernel).
@@ -92,6 +93,16 @@ int tma_smem_bytes(int vb, int np, int nmp);
 void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np,
                          int vb, int nsg, int grid, unsigned long long *prof, int n_prod, int tile_block,
                          size_t buf_off, cudaStream_t s);
+void pair_geom(int P, int n_v, int *np, int *n_ptiles, int *n_vtiles, int *n_tiles);
+int pair_list_cap(int max_L);
+size_t pair_entry_bytes();
+int pair_nsl(int np, int nmp);
+bool pair_supported(int P, int nmp);
+void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, size_t cnt_off,
+                       cudaStream_t s);
+void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, cudaStream_t s);
+void launch_pair_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np, int nsl,
+                      int grid, size_t buf_off, size_t cnt_off, cudaStream_t s);
 int persist_blocks_per_sm(int nmp, int np, int vb, int nsg, int n_prod);
 void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
 int persist_nsg(int np, int vb, int nmp);

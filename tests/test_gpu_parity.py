@@ -39,7 +39,7 @@ def _ctx_with_kernel(kernel):
             os.environ["MADPIPE_KERNEL"] = old
 
 
-@pytest.fixture(scope="module", params=["persist", "v1", "tma"])
+@pytest.fixture(scope="module", params=["pair", "persist", "v1", "tma"])
 def kctx(request):
     c = _ctx_with_kernel(request.param)
     yield c
@@ -250,7 +250,7 @@ def test_geometry_extremes(P, n_m, n_v, L):
     M = int((3 * ch["W"].sum() + 3 * ch["a"].sum()) * 0.6) + 1
     n_c = 9
     ref = oracle.solve(ch, P, M, 25.0, n_m, n_v, n_c, v_range=1, n_threads=4)
-    for kernel in ("persist", "v1", "tma"):
+    for kernel in ("pair", "persist", "v1", "tma"):
         c = _ctx_with_kernel(kernel)
         try:
             tau, root = c.candidates(ch, P, M, 25.0, n_m, n_v, n_c, v_range=1)
@@ -259,3 +259,33 @@ def test_geometry_extremes(P, n_m, n_v, L):
             _same_solution(got, ref)
         finally:
             c.close()
+
+
+@pytest.mark.parametrize("seed,P,n_m,n_v,L", [(11, 64, 8, 96, 24),    # 2 processor rows per thread
+                                              (12, 40, 4, 130, 18),   # ragged v-tiles, nmp 4
+                                              (13, 90, 8, 40, 15),    # 2 processor tiles (64 + 25)
+                                              (14, 33, 5, 200, 21)])  # odd n_m, one row past 32
+def test_two_layer_kernel_full_tables(seed, P, n_m, n_v, L):
+    """The two-layer step kernel (shared source rows, layer-(l+1) shift, the k = l+1
+    fixup) against the oracle's full tables, several candidates, both v ranges."""
+    rng = np.random.default_rng(seed)
+    ch = chaingen.tiny(rng, L)
+    M = int((3 * ch["W"].sum() + 3 * ch["a"].sum()) * 0.5) + 1
+    n_c = 6
+    c = _ctx_with_kernel("pair")
+    try:
+        for vr in (0, 1):
+            ref = oracle.solve(ch, P, M, 30.0, n_m, n_v, n_c, v_range=vr, n_threads=4)
+            tau, root = c.candidates(ch, P, M, 30.0, n_m, n_v, n_c, v_range=vr)
+            assert np.array_equal(tau, ref["tau"]) and np.array_equal(root, ref["root"]), vr
+            for j in (0, n_c // 2, n_c - 1):
+                A, ARG = c.dp_table(ch, P, M, 30.0, n_m, n_v, n_c, j=j, v_range=vr)
+                A_ref, ARG_ref, _ = oracle.table(ch, P, M, 30.0, n_m, n_v, vr, ref["tau"][j])
+                assert np.array_equal(A, A_ref), (vr, j)
+                assert np.array_equal(ARG, ARG_ref), (vr, j)
+            got = c.solve(ch, P, M, 30.0, n_m, n_v, n_c, v_range=vr)
+            _same_solution(got, ref)
+            sb = c.last_step_bytes()
+            assert sb["segments"] > 0 and sb["load_bytes"] > 0
+    finally:
+        c.close()
