@@ -43,6 +43,7 @@ struct madpipe_ctx {
     bool own_stream = false;
     int64_t mem_budget = 0;
     std::string err;
+    DevBuf tdesc;
     DevBuf tables, jobs, tiles, chains, chain_data, jl, counts, roots, trace, stages, scratch, codes, flags,
         tlist;
     cudaEvent_t ev_a = nullptr, ev_b = nullptr;
@@ -61,6 +62,8 @@ struct madpipe_ctx {
     int tile_block = 1;       // MADPIPE_TILE_BLOCK: consecutive tiles per interleaved block (1 = round-robin)
     DevBuf profbuf;
     int num_sms = 148;
+    int pair_overlap = 0;
+    // MADPIPE_PAIR_OVERLAP=1: pair_trans of the next pass on the aux stream
     int n_rec = 0;            // step-kernel launches bracketed by per-launch events in the last batch
     std::vector<cudaEvent_t> ev_pool;
 };
@@ -236,6 +239,7 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stre
     c->prof = pf && pf[0] == '1';
     if (const char *e = getenv("MADPIPE_NPROD")) c->n_prod = std::max(1, std::min(4, atoi(e)));
     if (const char *e = getenv("MADPIPE_TILE_BLOCK")) c->tile_block = std::max(1, atoi(e));
+    if (const char *e = getenv("MADPIPE_PAIR_OVERLAP")) c->pair_overlap = atoi(e) != 0;
     cudaEventCreate(&c->ev_a);
     cudaEventCreate(&c->ev_b);
     cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking);
@@ -253,6 +257,7 @@ extern "C" void madpipe_ctx_destroy(madpipe_ctx *c) {
     cudaSetDevice(c->device);
     cudaStreamSynchronize(c->stream);
     c->profbuf.release();
+    c->tdesc.release();
     DevBuf *bufs[] = {&c->tables, &c->jobs, &c->tiles, &c->chains, &c->chain_data, &c->jl,
                       &c->counts, &c->roots, &c->trace, &c->stages, &c->scratch, &c->codes, &c->flags, &c->tlist};
     for (DevBuf *b : bufs) b->release();
@@ -507,16 +512,23 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 n_v_max = std::max(n_v_max, J.n_v);
             }
             CUDA_TRY(ctx, ctx->tlist.ensure(2 * total * pair_entry_bytes()));
-            CUDA_TRY(ctx, ctx->codes.ensure(2 * vtotal * sizeof(int32_t)));
             list_buf_entries = total;
             cnt_buf_entries = vtotal;
             size_t off = 0, voff = 0, ftotal = 0, wtotal = 0;
+            // tile descriptors: (list offset of the tile's v-tile, processor tile)
+            std::vector<int32_t> hdesc(2 * htiles.size());
             for (auto &J : hjobs) {
                 int np_, npt_, nvt_, nt_;
                 pair_geom(J.P, J.n_v, &np_, &npt_, &nvt_, &nt_);
                 J.tlist = (TransEntry *)((char *)ctx->tlist.p + off * pair_entry_bytes());
-                J.tcount = (int32_t *)ctx->codes.p + voff;
+                J.tcount = nullptr;
                 J.code_cap = cap;
+                for (int vt = 0; vt < nvt_; vt++)
+                    for (int pt = 0; pt < npt_; pt++) {
+                        const size_t t = (size_t)J.tile0 + (size_t)vt * npt_ + pt;
+                        hdesc[2 * t] = (int32_t)(off + (size_t)vt * cap);
+                        hdesc[2 * t + 1] = pt;
+                    }
                 off += (size_t)nvt_ * (size_t)cap;
                 voff += (size_t)nvt_;
                 ftotal += (size_t)(J.L + 1) * (size_t)J.n_v;
@@ -531,6 +543,9 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 J.kwin = wbase + woff;
                 woff += (size_t)(J.L + 1);
             }
+            if (off > (size_t)INT32_MAX) return fail(ctx, MADPIPE_ENOMEM, "pair lists exceed 2^31 entries");
+            CUDA_TRY(ctx, ctx->tdesc.ensure(sizeof(int32_t) * hdesc.size()));
+            CUDA_TRY(ctx, h2d(ctx, ctx->tdesc.p, hdesc.data(), sizeof(int32_t) * hdesc.size()));
         }
         if (kern == 2) {
             // useful-transition lists of one layer: [job][v][maxL] entries + [job][v] counts
@@ -579,7 +594,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             p_np = hjobs[0].np;
             nsg = pair_nsl(p_np, nmp);
             if (nsg < 4) return fail(ctx, MADPIPE_EINVAL, "row segment too large for the pair step kernel ring");
-            persist_grid = std::min(n_tiles, ctx->num_sms);
+            persist_grid = std::min(n_tiles, ctx->num_sms * pair_blocks_per_sm(nmp, p_np, nsg));
         }
         if (kern == 2) {
             p_np = hjobs[0].np;
@@ -590,8 +605,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         }
         const bool per_launch = timed && ctx->per_launch_timing;
         if (ctx->prof) {
-            CUDA_TRY(ctx, ctx->profbuf.ensure(8 * sizeof(unsigned long long)));
-            CUDA_TRY(ctx, cudaMemsetAsync(ctx->profbuf.p, 0, 8 * sizeof(unsigned long long), ctx->stream));
+            CUDA_TRY(ctx, ctx->profbuf.ensure(16 * sizeof(unsigned long long)));
+            CUDA_TRY(ctx, cudaMemsetAsync(ctx->profbuf.p, 0, 16 * sizeof(unsigned long long), ctx->stream));
         }
         if (per_launch && ctx->ev_pool.size() < (size_t)(2 * maxL)) {
             while (ctx->ev_pool.size() < (size_t)(2 * maxL)) {
@@ -604,19 +619,42 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             launch_window(djobs, nj, maxL, ctx->stream);
             ctx->launches++;
             int n_rec = 0;
+            const int cap = pair_list_cap(maxL);
+            // pass i covers layers l = 2i+1, l+1 with list buffer i % 2.  pair_trans of
+            // pass i+1 runs on the aux stream, overlapping step + fixup of pass i: it
+            // waits for fixup of pass i-1 (flags of slabs <= l-1 final; its buffer,
+            // last read by step of pass i-1, free) and leaves slabs l, l+1 unverified.
+            launch_pair_trans(djobs, nj, n_v_max, 1, nmp, 0, 1, ctx->stream);
+            ctx->launches++;
+            CUDA_TRY(ctx, cudaEventRecord(ctx->ev_w, ctx->stream));
+            CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_w, 0));
+            const bool ov = ctx->pair_overlap != 0;
             for (int l = 1; l <= maxL; l += 2) {
-                const int b = (l >> 1) & 1;   // list buffer (double-buffered)
-                launch_pair_trans(djobs, nj, n_v_max, l, nmp, b * list_buf_entries, b * cnt_buf_entries, ctx->stream);
+                const int i = l >> 1, b = i & 1;
+                if (!ov && i >= 1) {
+                    launch_pair_trans(djobs, nj, n_v_max, l, nmp, (size_t)b * list_buf_entries, l, ctx->stream);
+                    ctx->launches++;
+                }
+                if (ov && l + 2 <= maxL) {
+                    if (i >= 1) CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_st[(i - 1) & 1], 0));
+                    launch_pair_trans(djobs, nj, n_v_max, l + 2, nmp, (size_t)(b ^ 1) * list_buf_entries, l, ctx->aux);
+                    CUDA_TRY(ctx, cudaEventRecord(ctx->ev_tr[(i + 1) & 1], ctx->aux));
+                    ctx->launches++;
+                }
+                if (ov && i >= 1) CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->stream, ctx->ev_tr[b], 0));
                 if (per_launch) cudaEventRecord(ctx->ev_pool[2 * n_rec], ctx->stream);
-                launch_pair_step(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, p_np, nsg, persist_grid,
-                                 b * list_buf_entries, b * cnt_buf_entries, ctx->stream);
+                launch_pair_step((const int2 *)ctx->tdesc.p, n_tiles, ctx->tlist.p, b * list_buf_entries, cap, nmp,
+                                 p_np, nsg, persist_grid,
+                                 (unsigned long long *)(ctx->prof ? ctx->profbuf.p : nullptr),
+                                 ctx->stream);
                 if (per_launch) cudaEventRecord(ctx->ev_pool[2 * n_rec + 1], ctx->stream);
                 n_rec++;
-                ctx->launches += 2;
+                ctx->launches++;
                 if (l + 1 <= maxL) {
                     launch_pair_fixup(djobs, nj, n_v_max, l + 1, nmp, ctx->stream);
                     ctx->launches++;
                 }
+                CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[b], ctx->stream));
             }
             ctx->n_rec = n_rec;
         } else {
@@ -658,6 +696,18 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         ctx->launches += 2;
         CUDA_TRY(ctx, cudaGetLastError());
         if (timed) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_b, ctx->stream));
+        if (ctx->prof && timed && kern == 3) {
+            unsigned long long pc[9];
+            CUDA_TRY(ctx, cudaMemcpy(pc, ctx->profbuf.p, sizeof pc, cudaMemcpyDeviceToHost));
+            const double g = (double)std::max(1, persist_grid);
+            fprintf(stderr,
+                    "[madpipe prof pair] batch of %d jobs, %d CTAs: producer %.3g cyc/CTA (empty waits %.1f%%, "
+                    "tile setup %.1f%%, push %.1f%%), %.3g tiles/CTA; consumer %.3g cyc/warp (queue waits %.1f%%, full waits "
+                    "%.1f%%), %.3g slot visits/warp\n",
+                    nj, persist_grid, pc[0] / g, 100.0 * pc[1] / std::max(1ull, pc[0]),
+                    100.0 * pc[2] / std::max(1ull, pc[0]), 100.0 * pc[8] / std::max(1ull, pc[0]), pc[7] / g, pc[3] / (g * 8),
+                    100.0 * pc[4] / std::max(1ull, pc[3]), 100.0 * pc[5] / std::max(1ull, pc[3]), pc[6] / (g * 8));
+        } else
         if (ctx->prof && timed) {
             unsigned long long pc[8];
             CUDA_TRY(ctx, cudaMemcpy(pc, ctx->profbuf.p, sizeof pc, cudaMemcpyDeviceToHost));

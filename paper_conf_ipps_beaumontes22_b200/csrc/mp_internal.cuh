@@ -98,11 +98,12 @@ int pair_list_cap(int max_L);
 size_t pair_entry_bytes();
 int pair_nsl(int np, int nmp);
 bool pair_supported(int P, int nmp);
-void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, size_t cnt_off,
+void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int unverified_from,
                        cudaStream_t s);
 void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, cudaStream_t s);
-void launch_pair_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np, int nsl,
-                      int grid, size_t buf_off, size_t cnt_off, cudaStream_t s);
+void launch_pair_step(const int2 *tdesc, int n_tiles, const void *lists, size_t buf_off, int cap, int nmp, int np,
+                      int nsl, int grid, unsigned long long *prof, cudaStream_t s);
+int pair_blocks_per_sm(int nmp, int np, int nsl);
 int persist_blocks_per_sm(int nmp, int np, int vb, int nsg, int n_prod);
 void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
 int persist_nsg(int np, int vb, int nmp);

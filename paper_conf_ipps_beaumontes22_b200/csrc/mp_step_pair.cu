@@ -67,25 +67,64 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t
         : "memory");
 }
 __device__ __forceinline__ double dmin(double a, double b) { return b < a ? b : a; }
+__device__ __forceinline__ void mbar_arrive_cnt(uint32_t bar, uint32_t cnt) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(cnt) : "memory");
+}
+// Queue publication inside one CTA: the producer warp's shared stores (queue
+// entry, then tail) are performed in program order by the shared-memory pipeline,
+// and the consumer polls the tail with volatile loads.  A release/acquire pair or
+// a fence here would also wait for the producer's outstanding global prefetch
+// loads (measured: ~35% of the producer's time), so plain volatile accesses are used.
+__device__ __forceinline__ void st_publish(int *p, int v) {
+    asm volatile("st.volatile.shared::cta.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+}
+__device__ __forceinline__ int ld_poll(const int *p) {
+    int v;
+    asm volatile("ld.volatile.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+    return v;
+}
 
 }  // namespace
 
-constexpr int kPairVB = 8;                       // delay rows per layer in a tile
+#ifndef MP_PAIR_VB
+#define MP_PAIR_VB 4
+#endif
+constexpr int kPairVB = MP_PAIR_VB;              // delay rows per layer in a tile
 constexpr int kPairRows = 2 * kPairVB;           // output rows (= consumer warps) per tile
-constexpr int kPairE = 2;                        // extra v-tiles: layer l+1 rows are shifted by <= kPairE*kPairVB
+constexpr int kPairE = 16 / kPairVB;             // extra v-tiles: layer l+1 rows are shifted by <= 16 levels
+constexpr int kPairCtas = 8 / kPairVB;           // resident CTAs per SM (one producer warp each)
 constexpr int kPairNp = 64;                      // processor rows per tile (2 per consumer thread)
-constexpr int kPairSlotsMax = 64;
+constexpr int kPairSlotsMax = 32;
 constexpr int kPairThreads = 32 * (kPairRows + 1);
+constexpr int kPairHdr = 2;                      // header entries at the head of each tile list
+constexpr int kPairStage = 32;                   // list head (header + 30 entries) prefetched per tile
 
 // One source row of a tile's merged list (pair_trans_kernel -> pair_step_kernel).
 struct PairEntry {
     uint16_t k;        // option k: the source is slab k-1
     uint16_t vp;       // next delay level v' (source row)
-    uint16_t mask;     // output rows of the tile that read it (bit r: r < 8 layer l, else l+1)
-    uint16_t pad;
-    uint8_t code[kPairRows];   // per row: d (bits 0-6, clamped to 127) | nf << 7
+    uint8_t mask;      // output rows of the tile that read it (bit r: r < 4 layer l, else l+1)
+    uint8_t pad[3];
+    uint8_t code[8];   // per row r < kPairRows: d (bits 0-6, clamped to 127) | nf << 7
+    double U0, U1;     // U(k,l), U(k,l+1)
 };
-static_assert(sizeof(PairEntry) == 24, "PairEntry size");
+static_assert(sizeof(PairEntry) == 32, "PairEntry size");
+
+// Tile header (the first kPairHdr entries of a tile list): what the producer
+// needs for the tile without reading the job descriptor.
+struct PairHdr {
+    int32_t n;         // entries
+    int32_t l;         // first layer of the pair
+    int32_t hasB;      // l+1 <= L
+    int32_t n_m;
+    double tau;
+    double *table;     // the job's DP table
+    uint32_t *flA;     // rowflag + l * n_v
+    int32_t n_v, P;
+    int32_t v0A, v0B;  // first delay row of layer l / layer l+1 in the tile
+    int64_t pad_;
+};
+static_assert(sizeof(PairHdr) == kPairHdr * sizeof(PairEntry), "PairHdr size");
 
 // delta of layer pair (l, l+1): layer l+1's rows of v-tile t are v0 - delta ..
 // (any delta is correct; this one maximises shared source rows).  Clamped so that
@@ -103,7 +142,11 @@ __device__ __forceinline__ int pair_vtiles(int n_v) { return (n_v + kPairVB - 1)
 // a3 + a4 for the layer pair (l, l+1).
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l, int nmp, size_t buf_off,
-                                                         size_t cnt_off) {
+                                                         int unverified_from) {
+    // unverified_from: source slabs >= this may still be being written by the pass
+    // this launch overlaps (step(l-2) + fixup(l-1)), so their row flags are not
+    // consulted -- those entries are kept (a read of an all-+inf row is harmless)
+    constexpr int KG = 32 / kPairRows;           // k values per warp iteration
     __shared__ Job sJ;
     if (threadIdx.x < sizeof(Job) / 8)
         reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
@@ -116,7 +159,7 @@ __global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l,
     if (vt >= pair_vtiles(J.n_v)) return;
     const bool hasB = l + 1 <= J.L;
     const int delta = pair_shift(J, l);
-    const int r = lane & 15, h = lane >> 4;      // row r of the tile; half h takes k = kb + h
+    const int r = lane % kPairRows, h = lane / kPairRows;   // row r of the tile; lane group h takes k = kb + h
     const bool isB = r >= kPairVB;
     const int lr = isB ? l + 1 : l;              // the row's layer
     const int v = isB ? vt * kPairVB - delta + (r - kPairVB) : vt * kPairVB + r;
@@ -124,6 +167,7 @@ __global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l,
     const size_t rowlen = (size_t)J.P * nmp;
     const size_t slab = (size_t)J.n_v * rowlen;
     const double Ulr = J.Up[lr];
+    const double Ul = J.Up[l], Ul1 = hasB ? J.Up[l + 1] : 0.0;
     // base row p = 0 (reading Q10) and the row flag, OR-ed later for p >= 1
     if (row_ok && h == 0) {
         const double U1l = __dsub_rn(Ulr, J.Up[0]);
@@ -139,8 +183,10 @@ __global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l,
     const int kw = isB ? (hasB ? J.kwin[l + 1] : l + 1) : kA;
     unsigned live = 0, useful = 0;
     int n = 0;
-    PairEntry *list = reinterpret_cast<PairEntry *>(J.tlist) + buf_off + (size_t)vt * J.code_cap;
-    for (int kb = kA; kb <= l; kb += 2) {        // k <= l: sources in slabs <= l-1 (final)
+    PairEntry *tl = reinterpret_cast<PairEntry *>(J.tlist) + buf_off + (size_t)vt * J.code_cap;
+    PairEntry *list = tl + kPairHdr;
+    const unsigned gmask = ((1u << kPairRows) - 1u) << (h * kPairRows);
+    for (int kb = kA; kb <= l; kb += KG) {       // k <= l: sources in slabs <= l-1 (final)
         const int k = kb + h;
         int key = -1 - lane;                     // unique unless the row reads a source
         uint32_t code = 0;
@@ -151,7 +197,7 @@ __global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l,
                 live++;
                 const int vn = tr & 0xFFFF;
                 // a source row that is +inf everywhere contributes +inf (exact skip)
-                if (J.rowflag[(size_t)(k - 1) * J.n_v + vn] != 0u) {
+                if (k - 1 >= unverified_from || J.rowflag[(size_t)(k - 1) * J.n_v + vn] != 0u) {
                     useful++;
                     key = (k << 16) | vn;
                     code = (uint32_t)(d > 127 ? 127 : d) | ((tr >> 24) & 1u) << 7;
@@ -165,14 +211,32 @@ __global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l,
         int idx = n + __popc(lb & ((1u << lane) - 1u));
         idx = __shfl_sync(0xffffffffu, idx, leader);
         if (lead) {
-            const uint64_t head = (uint64_t)(uint32_t)k | (uint64_t)(uint32_t)(key & 0xFFFF) << 16 |
-                                  (uint64_t)((grp >> (16 * h)) & 0xFFFFu) << 32;
-            *reinterpret_cast<uint64_t *>(list + idx) = head;
+            PairEntry *e = list + idx;
+            const double Uk = J.Up[k - 1];
+            *reinterpret_cast<uint64_t *>(e) = (uint64_t)(uint32_t)k | (uint64_t)(uint32_t)(key & 0xFFFF) << 16 |
+                                               (uint64_t)((grp & gmask) >> (h * kPairRows)) << 32;
+            e->U0 = __dsub_rn(Ul, Uk);
+            e->U1 = hasB ? __dsub_rn(Ul1, Uk) : 0.0;
         }
         if (key >= 0) list[idx].code[r] = (uint8_t)code;
         n += __popc(lb);
     }
-    if (lane == 0) J.tcount[cnt_off + vt] = n;
+    if (lane == 0) {
+        PairHdr hd;
+        hd.n = n;
+        hd.l = l;
+        hd.hasB = hasB ? 1 : 0;
+        hd.n_m = J.n_m;
+        hd.tau = J.tau;
+        hd.table = J.table;
+        hd.flA = J.rowflag + (size_t)l * J.n_v;
+        hd.n_v = J.n_v;
+        hd.P = J.P;
+        hd.v0A = vt * kPairVB;
+        hd.v0B = vt * kPairVB - delta;
+        hd.pad_ = 0;
+        *reinterpret_cast<PairHdr *>(tl) = hd;
+    }
     for (int o = 16; o > 0; o >>= 1) {
         live += __shfl_xor_sync(0xffffffffu, live, o);
         useful += __shfl_xor_sync(0xffffffffu, useful, o);
@@ -189,54 +253,56 @@ __global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l,
 // a5 for the layer pair: the persistent two-layer step kernel.
 // ---------------------------------------------------------------------------
 struct PairMeta {
-    uint32_t mask;          // rows reading this slot's source segment
     int16_t flags;          // 0 = data, 1 = tile end (store the rows), 4 = terminate
     int16_t np;             // processor rows of the tile
+    int32_t n_m;
     union {
         struct { double U0, U1; uint8_t code[kPairRows]; } e;       // data: U(k,l), U(k,l+1), codes
         struct { double tau; double *outA; uint32_t *flA; int32_t v0A, v0B; } t;  // tile end
     };
     int64_t slab;           // doubles per slab
     int32_t rowlen, n_v;
-    int32_t hasB, n_m;
+    int32_t hasB, pad_;
 };
 static_assert(sizeof(PairMeta) == 64, "PairMeta size");
 
-// relax one processor row of NMP levels held in lane-rotated chunk order
-// (same arithmetic and layout as step_persist_kernel's ROW mode)
+// relax one processor row of NMP levels held in lane-rotated chunk order (the
+// layout of step_persist_kernel's ROW mode: chunk c of a thread holds levels
+// 2j, 2j+1 with j = (c + rot) mod C, so a quarter-warp's 16-byte loads hit 8
+// distinct bank groups).  `off[c]` = byte offset of the thread's source row p-1,
+// chunk j, in the slot (precomputed once); S reads row p, levels m + d: the same
+// offset + NMP*8 + 8d.  S candidates with m + d > n_m - 1 are read (in bounds of
+// the padded ring) and discarded by predicate, so the code has no per-lane branch.
 template <int NMP>
-__device__ __forceinline__ void pair_relax(double (&best)[NMP], const double *rowN, int rot, int d, bool nf,
-                                           double U, int n_m) {
+__device__ __forceinline__ void pair_relax(double (&best)[NMP], const char *slot, const int (&off)[NMP / 2],
+                                           const int (&m2)[NMP / 2], int d, bool nf, double U, int lim) {
     constexpr int C = NMP / 2;
-    const double *rowS = rowN + NMP;
     if (nf) {                                                    // N
 #pragma unroll
         for (int c = 0; c < C; c++) {
-            const int j = (c + rot) & (C - 1);
-            const double2 x = *reinterpret_cast<const double2 *>(rowN + 2 * j);
+            const double2 x = *reinterpret_cast<const double2 *>(slot + off[c]);
             best[2 * c] = dmin(best[2 * c], x.x);
             best[2 * c + 1] = dmin(best[2 * c + 1], x.y);
         }
     }
-    if (d <= n_m - 1) {                                          // S
+    if (lim >= 0) {                                              // S: valid iff m <= lim = n_m-1-d
+        const char *srow = slot + NMP * 8 + 8 * d;
         if ((d & 1) == 0) {
-            const int e = d >> 1;
 #pragma unroll
             for (int c = 0; c < C; c++) {
-                const int j = (c + rot) & (C - 1);
-                if (2 * j + d <= n_m - 1) {
-                    const double2 y = *reinterpret_cast<const double2 *>(rowS + 2 * (j + e));
-                    best[2 * c] = dmin(best[2 * c], __dadd_rn(U, y.x));
-                    if (2 * j + 1 + d <= n_m - 1) best[2 * c + 1] = dmin(best[2 * c + 1], __dadd_rn(U, y.y));
-                }
+                const double2 y = *reinterpret_cast<const double2 *>(srow + off[c]);
+                const double c0 = __dadd_rn(U, y.x), c1 = __dadd_rn(U, y.y);
+                best[2 * c] = (m2[c] <= lim && c0 < best[2 * c]) ? c0 : best[2 * c];
+                best[2 * c + 1] = (m2[c] + 1 <= lim && c1 < best[2 * c + 1]) ? c1 : best[2 * c + 1];
             }
         } else {
 #pragma unroll
             for (int c = 0; c < C; c++) {
-                const int j = (c + rot) & (C - 1);
-                if (2 * j + d <= n_m - 1) best[2 * c] = dmin(best[2 * c], __dadd_rn(U, rowS[2 * j + d]));
-                if (2 * j + 1 + d <= n_m - 1)
-                    best[2 * c + 1] = dmin(best[2 * c + 1], __dadd_rn(U, rowS[2 * j + 1 + d]));
+                const double y0 = *reinterpret_cast<const double *>(srow + off[c]);
+                const double y1 = *reinterpret_cast<const double *>(srow + off[c] + 8);
+                const double c0 = __dadd_rn(U, y0), c1 = __dadd_rn(U, y1);
+                best[2 * c] = (m2[c] <= lim && c0 < best[2 * c]) ? c0 : best[2 * c];
+                best[2 * c + 1] = (m2[c] + 1 <= lim && c1 < best[2 * c + 1]) ? c1 : best[2 * c + 1];
             }
         }
     }
@@ -244,7 +310,7 @@ __device__ __forceinline__ void pair_relax(double (&best)[NMP], const double *ro
 
 // clamp (Q12) and store one processor row; returns whether a value is finite
 template <int NMP>
-__device__ __forceinline__ bool pair_store(double (&best)[NMP], double *o, int rot, double tau, int n_m) {
+__device__ __forceinline__ bool pair_store(const double (&best)[NMP], double *o, int rot, double tau, int n_m) {
     constexpr int C = NMP / 2;
     bool fin = false;
 #pragma unroll
@@ -256,31 +322,30 @@ __device__ __forceinline__ bool pair_store(double (&best)[NMP], double *o, int r
         fin |= (r.x <= tau) | (r.y <= tau);
         *reinterpret_cast<double2 *>(o + 2 * j) = r;
     }
-#pragma unroll
-    for (int i = 0; i < NMP; i++) best[i] = MP_INF;
     return fin;
 }
 
 template <int NMP>
-__global__ void __launch_bounds__(kPairThreads, 1) pair_step_kernel(const Job *__restrict__ jobs,
-                                                                    const int32_t *__restrict__ tile_job,
-                                                                    int n_tiles, int l, int np_max, int nsl,
-                                                                    int round, size_t buf_off, size_t cnt_off) {
+__global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(const int2 *__restrict__ tdesc, int n_tiles,
+                                                                    const PairEntry *__restrict__ lists,
+                                                                    int np_max, int nsl, int round,
+                                                                    int stage_n, unsigned long long *prof) {
     // Slots are shared by the rows that read them: the producer pushes each slot
     // (with the parity of its full-barrier phase) into the queue of every row in
     // its mask; a row warp visits only its own slots; the last reader (reference
     // count) releases the slot's empty barrier.  Tile ends and the final
-    // termination are slots without data pushed to all 16 rows.
+    // termination are slots without data pushed to all rows.  tdesc[tile] =
+    // (offset of the tile's list in `lists`, processor tile).
     constexpr int C = NMP / 2;
-    constexpr int QN = 64;                                 // queue entries per row (>= slots)
+    constexpr int QN = 32;                                 // queue entries per row (>= slots)
     extern __shared__ __align__(128) unsigned char dsm[];
     __shared__ __align__(8) uint64_t full[kPairSlotsMax];
     __shared__ __align__(8) uint64_t empty[kPairSlotsMax];
     __shared__ __align__(16) PairMeta meta[kPairSlotsMax];
-    __shared__ __align__(16) Job pJ;
-    __shared__ uint8_t rq[kPairRows][QN];                  // per-row queues: slot | phase parity << 7
+    __shared__ uint32_t rq[kPairRows][QN];                 // per-row queues: slot | parity << 6 | code << 16
     __shared__ int rtail[kPairRows];                       // entries pushed per row (producer)
-    __shared__ int sref[kPairSlotsMax];                    // readers left per slot
+    __shared__ __align__(128) PairEntry stage[2][kPairStage];   // list heads of this and the next tile
+    __shared__ __align__(8) uint64_t stbar[2];
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
@@ -290,107 +355,135 @@ __global__ void __launch_bounds__(kPairThreads, 1) pair_step_kernel(const Job *_
     if (tid == 0) {
         for (int s = 0; s < nsl; s++) {
             mbar_init(full0 + 8 * s, 1);
-            mbar_init(empty0 + 8 * s, 1);
+            mbar_init(empty0 + 8 * s, kPairRows);
         }
+        mbar_init(smem_u32(&stbar[0]), 1);
+        mbar_init(smem_u32(&stbar[1]), 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (tid < kPairRows) rtail[tid] = 0;
     __syncthreads();
-    const double *ring = reinterpret_cast<const double *>(dsm);
-    volatile int *vtail = rtail;
 
     if (warp == kPairRows) {
         // =========================================================== producer warp
-        int sl = 0, wraps = 0, cur = -1;
-        int my_tail = 0;                                   // lane r < 16: entries pushed to row r
+        int sl = 0, wraps = 0;
+        int tails[kPairRows];                              // entries pushed per row (same in every lane)
+#pragma unroll
+        for (int rr = 0; rr < kPairRows; rr++) tails[rr] = 0;
         const unsigned lt = (1u << lane) - 1u;
-        auto push = [&](bool act, uint32_t mask, uint32_t ent) {
-            // append ent to the queue of every row in mask, in lane order
+        auto push = [&](bool act, uint32_t mask, uint32_t ent, const uint8_t *codes) {
+            // append ent (+ the row's code) to the queue of every row in mask, in lane order
+            int mytail = 0;
 #pragma unroll
             for (int rr = 0; rr < kPairRows; rr++) {
                 const bool mine = act && ((mask >> rr) & 1u);
                 const unsigned bal = __ballot_sync(0xffffffffu, mine);
-                const int base = __shfl_sync(0xffffffffu, my_tail, rr);
-                if (mine) rq[rr][(base + __popc(bal & lt)) & (QN - 1)] = (uint8_t)ent;
-                if (lane == rr) my_tail += __popc(bal);
+                if (mine)
+                    reinterpret_cast<volatile uint32_t *>(rq[rr])[(tails[rr] + __popc(bal & lt)) & (QN - 1)] =
+                        ent | (uint32_t)codes[rr] << 16;
+                tails[rr] += __popc(bal);
+                if (lane == rr) mytail = tails[rr];
             }
             __syncwarp();
-            __threadfence_block();
-            if (lane < kPairRows) vtail[lane] = my_tail;
+            if (lane < kPairRows) st_publish(&rtail[lane], mytail);
         };
-        for (int tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
-            const int jid = tile_job[tile];
-            if (jid != cur) {
-                __syncwarp();
-                const uint64_t *src = reinterpret_cast<const uint64_t *>(jobs + jid);
-                uint64_t *dst = reinterpret_cast<uint64_t *>(&pJ);
-                for (int w = lane; w < (int)(sizeof(Job) / 8); w += 32) dst[w] = __ldg(src + w);
-                __syncwarp();
-                cur = jid;
-            }
-            const Job &J = pJ;
-            if (l > J.L) continue;
-            const int t = tile - J.tile0;
-            const int vt = t / J.n_ptiles, pt = t - (t / J.n_ptiles) * J.n_ptiles;
+        // prof (MADPIPE_PROF=1): [0] producer cycles, [1] empty-barrier waits (max over lanes),
+        // [2] tile setup (header), [3] consumer cycles, [4] queue waits, [5] full waits, [6] data
+        // slots consumed (row visits), [7] tiles
+        long long t_p0 = clock64(), t_we = 0, t_set = 0, n_tl = 0, t_push = 0;
+        // the head of each tile's list (header + first entries) is bulk-copied into a
+        // staging buffer one tile ahead, so a tile starts without a global-load round trip
+        const uint32_t st0 = smem_u32(&stbar[0]);
+        const uint32_t stage_bytes = (uint32_t)stage_n * (uint32_t)sizeof(PairEntry);
+        auto stage_copy = [&](int2 dsc, int buf) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive_expect_tx(st0 + 8 * buf, stage_bytes);
+            bulk_g2s(smem_u32(&stage[buf][0]), lists + dsc.x, stage_bytes, st0 + 8 * buf);
+        };
+        const int G = (int)gridDim.x;
+        int2 desc = blockIdx.x < n_tiles ? __ldg(tdesc + blockIdx.x) : make_int2(0, 0);
+        int2 nextd = (int)blockIdx.x + G < n_tiles ? __ldg(tdesc + blockIdx.x + G) : make_int2(0, 0);
+        if (lane == 0 && (int)blockIdx.x < n_tiles) stage_copy(desc, 0);
+        int it = 0;
+        for (int tile = blockIdx.x; tile < n_tiles; tile += G, it++) {
+            const long long t_t0 = prof ? clock64() : 0;
+            const int buf = it & 1;
+            if (lane == 0 && tile + G < n_tiles) stage_copy(nextd, buf ^ 1);
+            const int2 mine = desc;
+            desc = nextd;
+            nextd = tile + 2 * G < n_tiles ? __ldg(tdesc + tile + 2 * G) : make_int2(0, 0);
+            mbar_wait(st0 + 8 * buf, (uint32_t)((it >> 1) & 1));
+            const PairEntry *tl = lists + mine.x;
+            const PairEntry *sg = stage[buf];
+            const PairHdr hd = *reinterpret_cast<const PairHdr *>(sg);
+            auto entry = [&](int e) -> PairEntry { return e + kPairHdr < stage_n ? sg[kPairHdr + e] : tl[kPairHdr + e]; };
+            // first round's entries
+            PairEntry cur;
+            if (lane < round) cur = entry(lane);
+            const int pt = mine.y;
             const int p_lo = 1 + pt * np_max;
-            const int np = min(np_max, J.P - p_lo);
+            const int np = min(np_max, hd.P - p_lo);
             if (np <= 0) continue;
-            const bool hasB = l + 1 <= J.L;
-            const int delta = pair_shift(J, l);
-            const int64_t rowlen = (int64_t)J.P * NMP;
-            const int64_t slab = (int64_t)J.n_v * rowlen;
+            const int64_t rowlen = (int64_t)hd.P * NMP;
+            const int64_t slab = (int64_t)hd.n_v * rowlen;
             const uint32_t seg_bytes = (uint32_t)(np + 1) * NMP * 8u;
-            const int n = __ldg(J.tcount + cnt_off + vt);
-            const PairEntry *list = reinterpret_cast<const PairEntry *>(J.tlist) + buf_off + (size_t)vt * J.code_cap;
-            const double Ul = J.Up[l], Ul1 = hasB ? J.Up[l + 1] : 0.0;
+            const int n = hd.n;
             const int stages = n + 1;                      // entries, then the tile-end marker
+            if (prof) { t_set += clock64() - t_t0; n_tl++; }
             for (int r0 = 0; r0 < stages; r0 += round) {
                 const int q = r0 + lane;
                 const bool act = lane < round && q < stages;
+                PairEntry nxt;                             // prefetch the next round's entry
+                if (lane < round && q + round < n) nxt = entry(q + round);
                 uint32_t mask = 0, ent = 0;
+                uint8_t codes[kPairRows] = {};
                 if (act) {
                     int s = sl + lane, use = wraps;
                     if (s >= nsl) { s -= nsl; use++; }
+                    const long long tw = prof ? clock64() : 0;
                     if (use > 0) mbar_wait(empty0 + 8 * s, (uint32_t)((use - 1) & 1));
-                    ent = (uint32_t)s | (uint32_t)(use & 1) << 7;
+                    if (prof) {
+                        const unsigned dw = (unsigned)(clock64() - tw);
+                        const unsigned mx = __reduce_max_sync(__activemask(), dw);
+                        if (lane == 0) t_we += mx;
+                    }
+                    ent = (uint32_t)s | (uint32_t)(use & 1) << 6;
                     PairMeta &M = meta[s];
                     M.np = (int16_t)np;
-                    M.n_m = J.n_m;
+                    M.n_m = hd.n_m;
                     if (q < n) {
-                        const uint64_t *ep = reinterpret_cast<const uint64_t *>(list + q);
-                        const uint64_t head = __ldg(ep);
-                        const int k = (int)(head & 0xFFFFu), vp = (int)((head >> 16) & 0xFFFFu);
                         bulk_g2s(ring_s + 8u * (uint32_t)(s * seg_doubles),
-                                 J.table + (int64_t)(k - 1) * slab + (int64_t)vp * rowlen + (int64_t)(p_lo - 1) * NMP,
+                                 hd.table + (int64_t)(cur.k - 1) * slab + (int64_t)cur.vp * rowlen +
+                                     (int64_t)(p_lo - 1) * NMP,
                                  seg_bytes, full0 + 8 * s);
-                        mask = (uint32_t)(head >> 32) & 0xFFFFu;
-                        M.mask = mask;
+                        mask = cur.mask;
                         M.flags = 0;
-                        const double Uk = J.Up[k - 1];
-                        M.e.U0 = __dsub_rn(Ul, Uk);
-                        M.e.U1 = hasB ? __dsub_rn(Ul1, Uk) : 0.0;
-                        reinterpret_cast<uint64_t *>(M.e.code)[0] = __ldg(ep + 1);
-                        reinterpret_cast<uint64_t *>(M.e.code)[1] = __ldg(ep + 2);
-                        sref[s] = __popc(mask);
+                        M.e.U0 = cur.U0;
+                        M.e.U1 = cur.U1;
+#pragma unroll
+                        for (int rr = 0; rr < kPairRows; rr++) codes[rr] = cur.code[rr];
+                        // rows that do not read the slot release it now
+                        if (__popc(mask) < kPairRows) mbar_arrive_cnt(empty0 + 8 * s, kPairRows - __popc(mask));
                         mbar_arrive_expect_tx(full0 + 8 * s, seg_bytes);
                     } else {
                         mask = (1u << kPairRows) - 1u;
-                        M.mask = mask;
                         M.flags = 1;
-                        M.t.tau = J.tau;
-                        M.t.outA = J.table + (int64_t)l * slab + (int64_t)(vt * kPairVB) * rowlen + (int64_t)p_lo * NMP;
-                        M.t.flA = J.rowflag + (size_t)l * J.n_v;
-                        M.t.v0A = vt * kPairVB;
-                        M.t.v0B = vt * kPairVB - delta;
+                        M.t.tau = hd.tau;
+                        M.t.flA = hd.flA;
                         M.slab = slab;
                         M.rowlen = (int32_t)rowlen;
-                        M.n_v = J.n_v;
-                        M.hasB = hasB ? 1 : 0;
-                        sref[s] = kPairRows;
+                        M.n_v = hd.n_v;
+                        M.hasB = hd.hasB;
+                        M.t.v0A = hd.v0A;
+                        M.t.v0B = hd.v0B;
+                        M.t.outA = hd.table + (int64_t)hd.l * slab + (int64_t)hd.v0A * rowlen + (int64_t)p_lo * NMP;
                         mbar_arrive(full0 + 8 * s);
                     }
                 }
-                push(act, mask, ent);
+                const long long tpu = prof ? clock64() : 0;
+                push(act, mask, ent, codes);
+                if (prof && lane == 0) t_push += clock64() - tpu;
+                cur = nxt;
                 const int adv = min(round, stages - r0);
                 sl += adv;
                 if (sl >= nsl) { sl -= nsl; wraps++; }
@@ -402,36 +495,64 @@ __global__ void __launch_bounds__(kPairThreads, 1) pair_step_kernel(const Job *_
             if (act) {
                 if (wraps > 0) mbar_wait(empty0 + 8 * sl, (uint32_t)((wraps - 1) & 1));
                 meta[sl].flags = 4;
-                sref[sl] = kPairRows;
-                ent = (uint32_t)sl | (uint32_t)(wraps & 1) << 7;
+                ent = (uint32_t)sl | (uint32_t)(wraps & 1) << 6;
                 mbar_arrive(full0 + 8 * sl);
             }
-            push(act, (1u << kPairRows) - 1u, ent);
+            const uint8_t none[kPairRows] = {};
+            push(act, (1u << kPairRows) - 1u, ent, none);
+        }
+        if (prof && lane == 0) {
+            atomicAdd(prof + 0, (unsigned long long)(clock64() - t_p0));
+            atomicAdd(prof + 1, (unsigned long long)t_we);
+            atomicAdd(prof + 2, (unsigned long long)t_set);
+            atomicAdd(prof + 7, (unsigned long long)n_tl);
+            atomicAdd(prof + 8, (unsigned long long)t_push);
         }
         return;
     }
-
     // =============================================================== consumer warps
     const int r = warp;                                    // output row of the tile
     const bool isB = r >= kPairVB;
     constexpr int G8 = C >= 8 ? 1 : 8 / C;                 // lanes sharing a 128-byte window
     constexpr int RM = C >= 8 ? 8 : C;
     const int rot = (lane / G8) % RM;                      // lane + 32 has the same rotation
+    int off0[C], off1[C], m2[C];                           // chunk offsets of rows lane, lane+32
+#pragma unroll
+    for (int c = 0; c < C; c++) {
+        const int jj = (c + rot) & (C - 1);
+        m2[c] = 2 * jj;
+        off0[c] = (lane * NMP + 2 * jj) * 8;
+        off1[c] = ((lane + 32) * NMP + 2 * jj) * 8;
+    }
     double b0[NMP], b1[NMP];
 #pragma unroll
     for (int i = 0; i < NMP; i++) { b0[i] = MP_INF; b1[i] = MP_INF; }
+    const char *ring = reinterpret_cast<const char *>(dsm);
+    const int seg_bytes = seg_doubles * 8;
     int head = 0;
+    long long t_c0 = clock64(), t_q = 0, t_f = 0, n_sl = 0;
     for (;;) {
-        while (vtail[r] == head) { }
-        const uint32_t ent = reinterpret_cast<volatile uint8_t *>(rq[r])[head & (QN - 1)];
+        const long long ta = prof ? clock64() : 0;
+        while (ld_poll(&rtail[r]) == head) { }
+        const uint32_t ent = reinterpret_cast<volatile uint32_t *>(rq[r])[head & (QN - 1)];
         head++;
-        const int s = (int)(ent & 63u);
-        mbar_wait(full0 + 8 * s, (ent >> 7) & 1u);
+        const int s = (int)(ent & 63u);                    // this row's slot
+        const long long tb = prof ? clock64() : 0;
+        mbar_wait(full0 + 8 * s, (ent >> 6) & 1u);
+        if (prof) { const long long tc = clock64(); t_q += tb - ta; t_f += tc - tb; n_sl++; }
         const PairMeta &M = meta[s];
         const int flags = M.flags;
-        if (flags & 4) break;
-        const int np = M.np, n_m = M.n_m;
+        if (flags & 4) {
+            if (prof && lane == 0) {
+                atomicAdd(prof + 3, (unsigned long long)(clock64() - t_c0));
+                atomicAdd(prof + 4, (unsigned long long)t_q);
+                atomicAdd(prof + 5, (unsigned long long)t_f);
+                atomicAdd(prof + 6, (unsigned long long)n_sl);
+            }
+            break;
+        }
         if (flags & 1) {                                   // tile end: clamp (Q12), store, flag
+            const int np = M.np, n_m = M.n_m;
             const int v = isB ? M.t.v0B + (r - kPairVB) : M.t.v0A + r;
             const bool ok = (!isB || M.hasB) && v >= 0 && v < M.n_v;
             bool fin = false;
@@ -445,19 +566,18 @@ __global__ void __launch_bounds__(kPairThreads, 1) pair_step_kernel(const Job *_
 #pragma unroll
             for (int i = 0; i < NMP; i++) { b0[i] = MP_INF; b1[i] = MP_INF; }
         } else {
-            const uint32_t code = M.e.code[r];
-            const int d = (int)(code & 127u);
-            const bool nf = (code >> 7) & 1u;
+            // rows lane and lane+32 are relaxed whether or not they exist in this tile
+            // (np < 64): the extra rows read in-bounds ring bytes and are never stored
+            const int d = (int)((ent >> 16) & 127u);
+            const bool nf = (ent >> 23) & 1u;
             const double U = isB ? M.e.U1 : M.e.U0;
-            const double *base = ring + (size_t)s * seg_doubles;
-            if (lane < np) pair_relax<NMP>(b0, base + lane * NMP, rot, d, nf, U, n_m);
-            if (lane + 32 < np) pair_relax<NMP>(b1, base + (lane + 32) * NMP, rot, d, nf, U, n_m);
+            const int lim = M.n_m - 1 - d;
+            const char *slot = ring + s * seg_bytes;
+            pair_relax<NMP>(b0, slot, off0, m2, d, nf, U, lim);
+            pair_relax<NMP>(b1, slot, off1, m2, d, nf, U, lim);
         }
         __syncwarp();
-        if (lane == 0) {
-            __threadfence_block();
-            if (atomicSub(&sref[s], 1) == 1) mbar_arrive(empty0 + 8 * s);
-        }
+        if (lane == 0) mbar_arrive(empty0 + 8 * s);
     }
 }
 
@@ -520,43 +640,69 @@ void pair_geom(int P, int n_v, int *np, int *n_ptiles, int *n_vtiles, int *n_til
     *n_tiles = *n_vtiles * *n_ptiles;
 }
 
-int pair_list_cap(int max_L) { return kPairRows * (max_L > 0 ? max_L : 1); }
+int pair_list_cap(int max_L) { return kPairHdr + kPairRows * (max_L > 0 ? max_L : 1); }
 size_t pair_entry_bytes() { return sizeof(PairEntry); }
 
-// ring slots: as many as fit in ~200 KB
+// ring slots per CTA (2 CTAs per SM): as many as fit in ~100 KB
 int pair_nsl(int np, int nmp) {
     const int seg = (np + 1) * nmp * 8;
-    int slots = (200 * 1024) / seg;
+    int slots = (200 * 1024 / kPairCtas) / seg;
     return slots > kPairSlotsMax ? kPairSlotsMax : slots;
 }
 
 bool pair_supported(int P, int nmp) { return P >= 2 && (nmp == 4 || nmp == 8); }
 
-void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, size_t cnt_off,
+void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int unverified_from,
                        cudaStream_t s) {
     const int nvt = (n_v_max + kPairVB - 1) / kPairVB + kPairE;
-    pair_trans_kernel<<<dim3((nvt + 3) / 4, n_jobs), 128, 0, s>>>(jobs, l, nmp, buf_off, cnt_off);
+    pair_trans_kernel<<<dim3((nvt + 3) / 4, n_jobs), 128, 0, s>>>(jobs, l, nmp, buf_off, unverified_from);
 }
 
 void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, cudaStream_t s) {
     pair_fixup_kernel<<<dim3((n_v_max + 3) / 4, n_jobs), 128, 0, s>>>(jobs, l1, nmp);
 }
 
-void launch_pair_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np, int nsl,
-                      int grid, size_t buf_off, size_t cnt_off, cudaStream_t s) {
-    const int smem = nsl * (np + 1) * nmp * 8;
+static int pair_round(int nsl) {
     int round = nsl / 2;
     if (round > 32) round = 32;
-    if (round < 1) round = 1;
+    return round < 1 ? 1 : round;
+}
+
+static int pair_smem(int np, int nmp, int nsl) {
+    // slots of (np_max+1) rows; a thread of row 63 reads rows 63 and 64 (64 = the
+    // next slot), and S reads up to nmp levels further: pad one row + nmp levels
+    return (nsl * (kPairNp + 1) > 0 ? nsl * (np + 1) * nmp * 8 : 0) + (kPairNp + 2 - (np + 1)) * nmp * 8 + 2 * nmp * 8;
+}
+
+void launch_pair_step(const int2 *tdesc, int n_tiles, const void *lists, size_t buf_off, int cap, int nmp, int np,
+                      int nsl, int grid, unsigned long long *prof, cudaStream_t s) {
+    const int smem = pair_smem(np, nmp, nsl);
+    const int stage_n = cap < kPairStage ? cap : kPairStage;
+    const PairEntry *L = reinterpret_cast<const PairEntry *>(lists) + buf_off;
     switch (nmp) {
 #define MP_CASE(N)                                                                                     \
     case N:                                                                                            \
         cudaFuncSetAttribute(pair_step_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);   \
-        pair_step_kernel<N><<<grid, kPairThreads, smem, s>>>(jobs, tile_job, n_tiles, l, np, nsl, round, buf_off, cnt_off); \
+        pair_step_kernel<N><<<grid, kPairThreads, smem, s>>>(tdesc, n_tiles, L, np, nsl, pair_round(nsl), stage_n, prof); \
         break;
         MP_CASE(4) MP_CASE(8)
 #undef MP_CASE
     }
+}
+
+int pair_blocks_per_sm(int nmp, int np, int nsl) {
+    const int smem = pair_smem(np, nmp, nsl);
+    int n = 0;
+    switch (nmp) {
+#define MP_OCC(N)                                                                                      \
+    case N:                                                                                            \
+        cudaFuncSetAttribute(pair_step_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);   \
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, pair_step_kernel<N>, kPairThreads, smem);     \
+        break;
+        MP_OCC(4) MP_OCC(8)
+#undef MP_OCC
+    }
+    return n < 1 ? 1 : n;
 }
 
 }  // namespace mp
