@@ -28,6 +28,7 @@
 //                       thread owning processor rows p_lo+lane and p_lo+32+lane.
 //   pair_fixup_kernel : one warp per (job, v) of layer l+1: option k = l+1.
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 #include "mp_device.cuh"
@@ -664,6 +665,7 @@ void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp
 
 static int pair_round(int nsl) {
     int round = nsl / 2;
+    if (const char *e = getenv("MADPIPE_PAIR_ROUND")) round = atoi(e) < nsl ? atoi(e) : nsl;
     if (round > 32) round = 32;
     return round < 1 ? 1 : round;
 }
