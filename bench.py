@@ -208,7 +208,9 @@ def main():
             res, cu = solve_distributed(chain, *a, early_exit=early_exit, ctx=ctx, device=dev)
         t = ctx.last_timing()
         cnt = ctx.last_counts()
-        return res, cu, (cnt["effective_updates"], cnt["useful_updates"]), t["launches"], t["step_ms"]
+        sb = ctx.last_step_bytes()
+        return (res, cu, (cnt["effective_updates"], cnt["useful_updates"], sb["load_bytes"] + sb["store_bytes"]),
+                t["launches"], t["step_ms"])
 
     def timed(chain, k, early_exit=False):
         dev_ms, wall, cus, effs, launches, kern_ms, io = [], [], [], [], 0, 0.0, (0, 0)
@@ -281,8 +283,14 @@ def main():
     # algorithmic bytes: one fp64 source value per relaxation that must read the table:
     # a live transition (not skipped by delay overflow / C > tau / no fit) whose source row
     # holds a finite value; all-+inf rows and dead transitions read nothing
+    # algorithmic bytes of the step kernel: every source-row segment it must
+    # bring on chip (one per useful (k, v') of a tile; the two-layer kernel loads a row
+    # shared by its two layers once) plus every output row it stores; per GPU
+    kbytes_step = reduce(main_run["eff"][-1][2], SUM) / world
     units = useful_step if useful_step > 0 else eff_step
-    achieved = units * K * BYTES_PER_UPDATE / (kern_ms / 1e3) / 1e9 if kern_ms > 0 else None
+    achieved = kbytes_step * K / (kern_ms / 1e3) / 1e9 if kern_ms > 0 and kbytes_step > 0 else None
+    # what a kernel without cross-layer reuse would have to stream for the same relaxations
+    streaming = units / world * K * BYTES_PER_UPDATE / (kern_ms / 1e3) / 1e9 if kern_ms > 0 else None
     traffic = None
     prof = os.path.join(ROOT, "profiles", "step_kernel_traffic.json")
     if os.path.exists(prof):
@@ -308,12 +316,14 @@ def main():
         "useful_updates_per_step": useful_step,
         "result": {"cand_index": res["cand_index"], "period": res["period"],
                    "special_load": res["special_load"], "n_stages": len(res["stages"])},
-        "roofline": {"bound": "hbm", "kernel": "step_kernel", "achieved": achieved, "peak": hbm_peak,
+        "roofline": {"bound": "hbm", "kernel": ctx.last_kernel(), "achieved": achieved, "peak": hbm_peak,
                      "unit": "GB/s", "frac": (achieved / hbm_peak) if achieved else None,
                      "traffic": traffic, "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)",
-                     "bytes_per_update": BYTES_PER_UPDATE,
-                     "units": "useful relaxations (live transition, finite source row)"
-                     if useful_step > 0 else "effective relaxations",
+                     "algorithmic_bytes_per_step": kbytes_step,
+                     "bytes": "source-row segments loaded + output rows stored by the step kernel",
+                     "streaming_equiv": streaming,
+                     "streaming_equiv_units": "%d B x %s / step-kernel time" % (
+                         BYTES_PER_UPDATE, "useful relaxations" if useful_step > 0 else "effective relaxations"),
                      "kernel_share": kern_ms / tot_ms if tot_ms else None},
         "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(), "cpu_baseline": cpu,
     }

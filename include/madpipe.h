@@ -198,6 +198,12 @@ int madpipe_last_counts(const madpipe_ctx *ctx, int64_t *cell_updates, int64_t *
  * Host-computed from the device counters; no GPU access. */
 int madpipe_last_step_bytes(const madpipe_ctx *ctx, int64_t *load_bytes, int64_t *store_bytes,
                             int64_t *segments);
+/* Step kernel that ran the largest batch of the last sweep:
+ * 0 = plain-load step_kernel, 1 = per-tile TMA step_tma_kernel, 2 = persistent
+ * single-layer step_persist_kernel, 3 = persistent two-layer pair_step_kernel.
+ * Chosen per batch from the row-segment size unless MADPIPE_KERNEL forces one.
+ * Host only. */
+int madpipe_last_kernel(const madpipe_ctx *ctx, int32_t *kernel);
 
 /* ---- NEXT row f2: the 1F1B* pattern of a contiguous allocation (host only) --
  * For stages s_1..s_N (one per GPU, tiling layers 1..L in order; e.g. a

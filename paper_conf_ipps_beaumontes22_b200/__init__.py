@@ -238,6 +238,13 @@ class Context:
         N.check(self._lib.madpipe_last_step_bytes(self.h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)))
         return dict(load_bytes=a.value, store_bytes=b.value, segments=c.value)
 
+    def last_kernel(self):
+        """Step kernel of the largest batch of the last sweep (madpipe_last_kernel)."""
+        k = ctypes.c_int32()
+        N.check(self._lib.madpipe_last_kernel(self.h, ctypes.byref(k)))
+        return {0: "step_kernel", 1: "step_tma_kernel", 2: "step_persist_kernel",
+                3: "pair_step_kernel"}.get(k.value, None)
+
     def last_timing(self):
         s = ctypes.c_double(); k = ctypes.c_double(); n = ctypes.c_int64()
         N.check(self._lib.madpipe_last_timing(self.h, ctypes.byref(s), ctypes.byref(k), ctypes.byref(n)))

@@ -9,7 +9,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libmadpipe.so")
+# MADPIPE_LIB: an alternative in-tree build (A/B experiments, build.py MADPIPE_DEFS)
+LIB_PATH = os.environ.get("MADPIPE_LIB") or os.path.join(_HERE, "libmadpipe.so")
 
 OK, INFEASIBLE, EINVAL, ENOMEM, ECUDA, ESTATE = 0, 1, -1, -2, -3, -5
 VRANGE_PAPER, VRANGE_SAFE = 0, 1
@@ -83,6 +84,7 @@ def lib():
         "madpipe_last_io": (ctypes.c_int, [vp, _i64p, _i64p]),
         "madpipe_last_counts": (ctypes.c_int, [vp, _i64p, _i64p, _i64p]),
         "madpipe_last_step_bytes": (ctypes.c_int, [vp, _i64p, _i64p, _i64p]),
+        "madpipe_last_kernel": (ctypes.c_int, [vp, _i32p]),
         "madpipe_solve_paper": (ctypes.c_int, [vp, cp, ctypes.c_int32, ctypes.c_int64, ctypes.c_double,
                                                ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ap,
                                                _dp, _dp]),
@@ -104,7 +106,7 @@ EXPORTED = ["madpipe_ctx_create", "madpipe_ctx_destroy", "madpipe_last_error", "
             "madpipe_shard", "madpipe_cell_updates", "madpipe_solve", "madpipe_solve_dev",
             "madpipe_sweep", "madpipe_resolve", "madpipe_solve_batch", "madpipe_candidates",
             "madpipe_dp_table", "madpipe_last_timing", "madpipe_set_timing", "madpipe_last_io",
-            "madpipe_last_counts", "madpipe_last_step_bytes", "madpipe_schedule", "madpipe_solve_paper", "madpipe_literal_table"]
+            "madpipe_last_counts", "madpipe_last_step_bytes", "madpipe_last_kernel", "madpipe_schedule", "madpipe_solve_paper", "madpipe_literal_table"]
 
 
 class MadpipeError(RuntimeError):

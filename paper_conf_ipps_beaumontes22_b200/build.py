@@ -13,13 +13,13 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-LIB = os.path.join(HERE, "libmadpipe.so")
+LIB = os.environ.get("MADPIPE_LIB") or os.path.join(HERE, "libmadpipe.so")
 SOURCES = ["mp_kernels.cu", "mp_step_tma.cu", "mp_step_persist.cu", "mp_step_pair.cu", "mp_api.cu", "mp_schedule.cu", "mp_literal.cu"]
 HEADERS = ["mp_internal.cuh", "mp_device.cuh", os.path.join("..", "..", "include", "madpipe.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "--fmad=false", "-Xcompiler", "-fPIC,-ffp-contract=off",
-         "-Xptxas", "-v"]
+         "-Xptxas", "-v"] + os.environ.get("MADPIPE_DEFS", "").split()   # A/B experiment macros
 
 
 def _stale() -> bool:
@@ -35,7 +35,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     objs = []
     for src in SOURCES:
-        obj = os.path.join(CSRC, src.replace(".cu", ".o"))
+        obj = LIB + "." + src.replace(".cu", ".o")
         cmd = [NVCC, *ARCH, *FLAGS, "-c", os.path.join(CSRC, src), "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:

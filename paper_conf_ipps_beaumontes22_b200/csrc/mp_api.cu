@@ -65,6 +65,8 @@ struct madpipe_ctx {
     int pair_overlap = 0;
     // MADPIPE_PAIR_OVERLAP=1: pair_trans of the next pass on the aux stream
     int n_rec = 0;            // step-kernel launches bracketed by per-launch events in the last batch
+    int last_kernel = -1;     // step kernel of the largest batch of the last timed sweep
+    int last_kernel_jobs = 0;
     std::vector<cudaEvent_t> ev_pool;
 };
 
@@ -301,6 +303,12 @@ extern "C" int madpipe_last_step_bytes(const madpipe_ctx *c, int64_t *load_bytes
     return MADPIPE_OK;
 }
 
+extern "C" int madpipe_last_kernel(const madpipe_ctx *c, int32_t *kernel) {
+    if (!c || !kernel) return MADPIPE_EINVAL;
+    *kernel = c->last_kernel;
+    return MADPIPE_OK;
+}
+
 extern "C" int madpipe_last_io(const madpipe_ctx *c, int64_t *h2d_bytes, int64_t *d2h_bytes) {
     if (!c) return MADPIPE_EINVAL;
     if (h2d_bytes) *h2d_bytes = c->h2d_bytes;
@@ -417,6 +425,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
     if (timed) {
         ctx->sweep_ms = 0.0; ctx->step_ms = 0.0;
         ctx->last_cell_updates = 0; ctx->last_effective = 0; ctx->last_useful = 0; ctx->last_segs = 0;
+        ctx->last_kernel = -1; ctx->last_kernel_jobs = 0;
         ctx->last_load_bytes = 0; ctx->last_store_bytes = 0;
     }
     std::vector<Job> hjobs;
@@ -434,7 +443,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         // one row segment per stage, which pays off from ~1 KB segments; below, plain loads win
         int kern = ctx->kernel;
         while (next < js.size() && early_exit && jl_host[js[next].chain] < js[next].j) next++;
-        if (kern == 3 && next < js.size() && !pair_supported(cs[js[next].chain].P, nmp)) kern = -1;
+        if (kern == 3 && next < js.size() && !pair_supported(cs[js[next].chain].P, nmp, disc->n_delay)) kern = -1;
         if (kern < 0 && next < js.size()) {
             int vb_, np_, npt_, nt_;
             persist_geom(cs[js[next].chain].P, disc->n_delay, nmp, &vb_, &np_, &npt_, &nt_);
@@ -698,7 +707,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         if (timed) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_b, ctx->stream));
         if (ctx->prof && timed && kern == 3) {
             unsigned long long pc[9];
-            CUDA_TRY(ctx, cudaMemcpy(pc, ctx->profbuf.p, sizeof pc, cudaMemcpyDeviceToHost));
+            CUDA_TRY(ctx, cudaMemcpyAsync(pc, ctx->profbuf.p, sizeof pc, cudaMemcpyDeviceToHost, ctx->stream));
+            CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
             const double g = (double)std::max(1, persist_grid);
             fprintf(stderr,
                     "[madpipe prof pair] batch of %d jobs, %d CTAs: producer %.3g cyc/CTA (empty waits %.1f%%, "
@@ -710,7 +720,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         } else
         if (ctx->prof && timed) {
             unsigned long long pc[8];
-            CUDA_TRY(ctx, cudaMemcpy(pc, ctx->profbuf.p, sizeof pc, cudaMemcpyDeviceToHost));
+            CUDA_TRY(ctx, cudaMemcpyAsync(pc, ctx->profbuf.p, sizeof pc, cudaMemcpyDeviceToHost, ctx->stream));
+            CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
             fprintf(stderr,
                     "[madpipe prof] batch of %d jobs, %d CTAs: producer total %.3g cyc/CTA: setup %.1f%% "
                     "lists %.1f%% issue %.1f%% (empty waits %.1f%%); consumer warp0 waits on full %.1f%%; "
@@ -748,6 +759,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 ctx->last_store_bytes += (int64_t)J.L * J.n_v * (J.P - 1) * rowb;
             }
         }
+        if (timed && nj > ctx->last_kernel_jobs) { ctx->last_kernel = kern; ctx->last_kernel_jobs = nj; }
         if (timed) {
             float ms = 0.f;
             cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b);

@@ -112,7 +112,8 @@ struct PairEntry {
 static_assert(sizeof(PairEntry) == 32, "PairEntry size");
 
 // Tile header (the first kPairHdr entries of a tile list): what the producer
-// needs for the tile without reading the job descriptor.
+// needs for the tile without reading the job descriptor.  n < 0: the job has no
+// layer l (l > L in a batch of chains of different lengths): the tile is skipped.
 struct PairHdr {
     int32_t n;         // entries
     int32_t l;         // first layer of the pair
@@ -154,10 +155,15 @@ __global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l,
             __ldg(reinterpret_cast<const uint64_t *>(jobs + blockIdx.y) + threadIdx.x);
     __syncthreads();
     const Job &J = sJ;
-    if (l > J.L) return;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int vt = blockIdx.x * 4 + warp;
     if (vt >= pair_vtiles(J.n_v)) return;
+    if (l > J.L) {                               // no layer l (a shorter chain of the batch):
+        if (lane == 0)                           // the step kernel skips the tile
+            reinterpret_cast<PairHdr *>(reinterpret_cast<PairEntry *>(J.tlist) + buf_off +
+                                        (size_t)vt * J.code_cap)->n = -1;
+        return;
+    }
     const bool hasB = l + 1 <= J.L;
     const int delta = pair_shift(J, l);
     const int r = lane % kPairRows, h = lane / kPairRows;   // row r of the tile; lane group h takes k = kb + h
@@ -417,6 +423,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             const PairEntry *tl = lists + mine.x;
             const PairEntry *sg = stage[buf];
             const PairHdr hd = *reinterpret_cast<const PairHdr *>(sg);
+            if (hd.n < 0) continue;                       // the job has no layer l
             auto entry = [&](int e) -> PairEntry { return e + kPairHdr < stage_n ? sg[kPairHdr + e] : tl[kPairHdr + e]; };
             // first round's entries
             PairEntry cur;
@@ -651,7 +658,7 @@ int pair_nsl(int np, int nmp) {
     return slots > kPairSlotsMax ? kPairSlotsMax : slots;
 }
 
-bool pair_supported(int P, int nmp) { return P >= 2 && (nmp == 4 || nmp == 8); }
+bool pair_supported(int P, int nmp, int n_v) { return P >= 2 && (nmp == 4 || nmp == 8) && n_v <= 65535; }
 
 void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int unverified_from,
                        cudaStream_t s) {

@@ -289,3 +289,24 @@ def test_two_layer_kernel_full_tables(seed, P, n_m, n_v, L):
             assert sb["segments"] > 0 and sb["load_bytes"] > 0
     finally:
         c.close()
+
+
+@pytest.mark.parametrize("kernel", ["pair", "persist", "v1"])
+def test_batch_mixed_lengths(kernel):
+    """One solve_batch over chains of different lengths and one P (they share a
+    launch): passes beyond a chain's L must leave its table alone, for every step
+    kernel; each chain's solution equals the oracle's."""
+    rng = np.random.default_rng(77)
+    Ls = [9, 23, 4, 16, 31, 12]
+    chains = [chaingen.tiny(rng, L) for L in Ls]
+    P, n_m, n_v, n_c = 40, 8, 48, 7
+    Ms = [int((3 * ch["W"].sum() + 3 * ch["a"].sum()) * 0.5) + 1 for ch in chains]
+    Bs = [30.0] * len(chains)
+    c = _ctx_with_kernel(kernel)
+    try:
+        res = c.solve_batch(chains, [P] * len(chains), Ms, Bs, n_m, n_v, n_c, v_range=1)
+    finally:
+        c.close()
+    for ch, M, got in zip(chains, Ms, res):
+        ref = oracle.solve(ch, P, M, 30.0, n_m, n_v, n_c, v_range=1, n_threads=4)
+        _same_solution(got, ref)
