@@ -98,7 +98,13 @@ constexpr int kPairNp = 64;                      // processor rows per tile (2 p
 constexpr int kPairSlotsMax = 32;
 constexpr int kPairThreads = 32 * (kPairRows + 1);
 constexpr int kPairHdr = 2;                      // header entries at the head of each tile list
-constexpr int kPairStage = 32;                   // list head (header + 30 entries) prefetched per tile
+#ifndef MP_POLL_NS
+#define MP_POLL_NS 100
+#endif
+#ifndef MP_PAIR_STAGE
+#define MP_PAIR_STAGE 32
+#endif
+constexpr int kPairStage = MP_PAIR_STAGE;        // list head (header + entries) prefetched per tile
 
 // One source row of a tile's merged list (pair_trans_kernel -> pair_step_kernel).
 struct PairEntry {
@@ -193,40 +199,59 @@ __global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l,
     PairEntry *tl = reinterpret_cast<PairEntry *>(J.tlist) + buf_off + (size_t)vt * J.code_cap;
     PairEntry *list = tl + kPairHdr;
     const unsigned gmask = ((1u << kPairRows) - 1u) << (h * kPairRows);
-    for (int kb = kA; kb <= l; kb += KG) {       // k <= l: sources in slabs <= l-1 (final)
-        const int k = kb + h;
-        int key = -1 - lane;                     // unique unless the row reads a source
-        uint32_t code = 0;
-        if (row_ok && k <= l && k >= kw) {
-            int64_t d;
-            const int32_t tr = transition(J, k, lr, v, __dsub_rn(Ulr, J.Up[k - 1]), &d);
-            if (tr >= 0) {
-                live++;
-                const int vn = tr & 0xFFFF;
-                // a source row that is +inf everywhere contributes +inf (exact skip)
-                if (k - 1 >= unverified_from || J.rowflag[(size_t)(k - 1) * J.n_v + vn] != 0u) {
-                    useful++;
-                    key = (k << 16) | vn;
-                    code = (uint32_t)(d > 127 ? 127 : d) | ((tr >> 24) & 1u) << 7;
+    // k <= l: sources in slabs <= l-1 (final).  TU k-groups per chunk: their transitions
+    // (independent global loads) and then their row flags are fetched together, so a
+    // chunk costs two memory round trips instead of two per k-group.
+    constexpr int TU = 4;
+    for (int kc = kA; kc <= l; kc += KG * TU) {
+        int key[TU];
+        uint32_t code[TU];
+#pragma unroll
+        for (int u = 0; u < TU; u++) {
+            const int k = kc + u * KG + h;
+            key[u] = -1 - lane;                  // unique unless the row reads a source
+            code[u] = 0;
+            if (row_ok && k <= l && k >= kw) {
+                int64_t d;
+                const int32_t tr = transition(J, k, lr, v, __dsub_rn(Ulr, J.Up[k - 1]), &d);
+                if (tr >= 0) {
+                    live++;
+                    key[u] = (k << 16) | (tr & 0xFFFF);
+                    code[u] = (uint32_t)(d > 127 ? 127 : d) | ((tr >> 24) & 1u) << 7;
                 }
             }
         }
-        const unsigned grp = __match_any_sync(0xffffffffu, key);
-        const int leader = __ffs(grp) - 1;
-        const bool lead = key >= 0 && leader == lane;
-        const unsigned lb = __ballot_sync(0xffffffffu, lead);
-        int idx = n + __popc(lb & ((1u << lane) - 1u));
-        idx = __shfl_sync(0xffffffffu, idx, leader);
-        if (lead) {
-            PairEntry *e = list + idx;
-            const double Uk = J.Up[k - 1];
-            *reinterpret_cast<uint64_t *>(e) = (uint64_t)(uint32_t)k | (uint64_t)(uint32_t)(key & 0xFFFF) << 16 |
-                                               (uint64_t)((grp & gmask) >> (h * kPairRows)) << 32;
-            e->U0 = __dsub_rn(Ul, Uk);
-            e->U1 = hasB ? __dsub_rn(Ul1, Uk) : 0.0;
+        uint32_t fl[TU];
+#pragma unroll
+        for (int u = 0; u < TU; u++) {
+            const int k = key[u] >> 16;
+            fl[u] = 1u;
+            if (key[u] >= 0 && k - 1 < unverified_from)
+                fl[u] = J.rowflag[(size_t)(k - 1) * J.n_v + (key[u] & 0xFFFF)];
         }
-        if (key >= 0) list[idx].code[r] = (uint8_t)code;
-        n += __popc(lb);
+#pragma unroll
+        for (int u = 0; u < TU; u++) {
+            // a source row that is +inf everywhere contributes +inf (exact skip)
+            if (key[u] >= 0 && fl[u] == 0u) key[u] = -1 - lane;
+            if (key[u] >= 0) useful++;
+            const unsigned grp = __match_any_sync(0xffffffffu, key[u]);
+            const int leader = __ffs(grp) - 1;
+            const bool lead = key[u] >= 0 && leader == lane;
+            const unsigned lb = __ballot_sync(0xffffffffu, lead);
+            int idx = n + __popc(lb & ((1u << lane) - 1u));
+            idx = __shfl_sync(0xffffffffu, idx, leader);
+            if (lead) {
+                const int k = key[u] >> 16;
+                PairEntry *e = list + idx;
+                const double Uk = J.Up[k - 1];
+                *reinterpret_cast<uint64_t *>(e) = (uint64_t)(uint32_t)k | (uint64_t)(uint32_t)(key[u] & 0xFFFF) << 16 |
+                                                   (uint64_t)((grp & gmask) >> (h * kPairRows)) << 32;
+                e->U0 = __dsub_rn(Ul, Uk);
+                e->U1 = hasB ? __dsub_rn(Ul1, Uk) : 0.0;
+            }
+            if (key[u] >= 0) list[idx].code[r] = (uint8_t)code[u];
+            n += __popc(lb);
+        }
     }
     if (lane == 0) {
         PairHdr hd;
@@ -378,7 +403,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
 #pragma unroll
         for (int rr = 0; rr < kPairRows; rr++) tails[rr] = 0;
         const unsigned lt = (1u << lane) - 1u;
-        auto push = [&](bool act, uint32_t mask, uint32_t ent, const uint8_t *codes) {
+        auto push = [&](bool act, uint32_t mask, uint32_t ent, uint64_t codes) {   // codes: byte rr = row rr
             // append ent (+ the row's code) to the queue of every row in mask, in lane order
             int mytail = 0;
 #pragma unroll
@@ -387,7 +412,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 const unsigned bal = __ballot_sync(0xffffffffu, mine);
                 if (mine)
                     reinterpret_cast<volatile uint32_t *>(rq[rr])[(tails[rr] + __popc(bal & lt)) & (QN - 1)] =
-                        ent | (uint32_t)codes[rr] << 16;
+                        ent | (uint32_t)((codes >> (8 * rr)) & 0xFFu) << 16;
                 tails[rr] += __popc(bal);
                 if (lane == rr) mytail = tails[rr];
             }
@@ -444,7 +469,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 PairEntry nxt;                             // prefetch the next round's entry
                 if (lane < round && q + round < n) nxt = entry(q + round);
                 uint32_t mask = 0, ent = 0;
-                uint8_t codes[kPairRows] = {};
+                uint64_t codes = 0;                         // in a register (an array was spilled)
                 if (act) {
                     int s = sl + lane, use = wraps;
                     if (s >= nsl) { s -= nsl; use++; }
@@ -468,8 +493,8 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                         M.flags = 0;
                         M.e.U0 = cur.U0;
                         M.e.U1 = cur.U1;
-#pragma unroll
-                        for (int rr = 0; rr < kPairRows; rr++) codes[rr] = cur.code[rr];
+                        static_assert(kPairRows <= 8, "codes packing");
+                        codes = *reinterpret_cast<const uint64_t *>(cur.code);
                         // rows that do not read the slot release it now
                         if (__popc(mask) < kPairRows) mbar_arrive_cnt(empty0 + 8 * s, kPairRows - __popc(mask));
                         mbar_arrive_expect_tx(full0 + 8 * s, seg_bytes);
@@ -506,8 +531,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 ent = (uint32_t)sl | (uint32_t)(wraps & 1) << 6;
                 mbar_arrive(full0 + 8 * sl);
             }
-            const uint8_t none[kPairRows] = {};
-            push(act, (1u << kPairRows) - 1u, ent, none);
+            push(act, (1u << kPairRows) - 1u, ent, 0ull);
         }
         if (prof && lane == 0) {
             atomicAdd(prof + 0, (unsigned long long)(clock64() - t_p0));
@@ -541,7 +565,13 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     long long t_c0 = clock64(), t_q = 0, t_f = 0, n_sl = 0;
     for (;;) {
         const long long ta = prof ? clock64() : 0;
-        while (ld_poll(&rtail[r]) == head) { }
+        // an empty queue: back off instead of spinning (a spinning warp takes issue slots
+        // from the producer and the working rows)
+        while (ld_poll(&rtail[r]) == head) {
+#if MP_POLL_NS > 0
+            __nanosleep(MP_POLL_NS);
+#endif
+        }
         const uint32_t ent = reinterpret_cast<volatile uint32_t *>(rq[r])[head & (QN - 1)];
         head++;
         const int s = (int)(ent & 63u);                    // this row's slot
