@@ -63,8 +63,6 @@ struct madpipe_ctx {
     int tile_block = 1;       // MADPIPE_TILE_BLOCK: consecutive tiles per interleaved block (1 = round-robin)
     DevBuf profbuf;
     int num_sms = 148;
-    int pair_overlap = 0;
-    // MADPIPE_PAIR_OVERLAP=1: pair_trans of the next pass on the aux stream
     int n_rec = 0;            // step-kernel launches bracketed by per-launch events in the last batch
     int last_kernel = -1;     // step kernel of the largest batch of the last timed sweep
     int last_kernel_jobs = 0;
@@ -242,7 +240,6 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stre
     c->prof = pf && pf[0] == '1';
     if (const char *e = getenv("MADPIPE_NPROD")) c->n_prod = std::max(1, std::min(4, atoi(e)));
     if (const char *e = getenv("MADPIPE_TILE_BLOCK")) c->tile_block = std::max(1, atoi(e));
-    if (const char *e = getenv("MADPIPE_PAIR_OVERLAP")) c->pair_overlap = atoi(e) != 0;
     cudaEventCreate(&c->ev_a);
     cudaEventCreate(&c->ev_b);
     cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking);
@@ -634,28 +631,18 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             ctx->launches++;
             int n_rec = 0;
             const int cap = pair_list_cap(maxL);
-            // pass i covers layers l = 2i+1, l+1 with list buffer i % 2.  pair_trans of
-            // pass i+1 runs on the aux stream, overlapping step + fixup of pass i: it
-            // waits for fixup of pass i-1 (flags of slabs <= l-1 final; its buffer,
-            // last read by step of pass i-1, free) and leaves slabs l, l+1 unverified.
-            launch_pair_trans(djobs, nj, n_v_max, 1, nmp, 0, 1, ctx->stream);
+            // pass i covers layers l = 2i+1, l+1 with list buffer i % 2:
+            //   stream: [wait trans(i)] step(i) -> fixup(i)
+            //   aux:    [wait step(i)]  trans(i+1)
+            // trans(i+1) writes list buffer (i+1) % 2 (last read by step(i-1)), reads the
+            // final flags of slabs <= l and, for slab l+1, a superset of what fixup(i)
+            // will flag (pair_trans_kernel, fix_slab).  (Measured: the two kernels hardly
+            // overlap, and one launch with their blocks interleaved was slower, 6.3.)
+            launch_pair_trans(djobs, nj, n_v_max, 1, nmp, 0, -1, ctx->stream);
             ctx->launches++;
-            CUDA_TRY(ctx, cudaEventRecord(ctx->ev_w, ctx->stream));
-            CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_w, 0));
-            const bool ov = ctx->pair_overlap != 0;
             for (int l = 1; l <= maxL; l += 2) {
                 const int i = l >> 1, b = i & 1;
-                if (!ov && i >= 1) {
-                    launch_pair_trans(djobs, nj, n_v_max, l, nmp, (size_t)b * list_buf_entries, l, ctx->stream);
-                    ctx->launches++;
-                }
-                if (ov && l + 2 <= maxL) {
-                    if (i >= 1) CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_st[(i - 1) & 1], 0));
-                    launch_pair_trans(djobs, nj, n_v_max, l + 2, nmp, (size_t)(b ^ 1) * list_buf_entries, l, ctx->aux);
-                    CUDA_TRY(ctx, cudaEventRecord(ctx->ev_tr[(i + 1) & 1], ctx->aux));
-                    ctx->launches++;
-                }
-                if (ov && i >= 1) CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->stream, ctx->ev_tr[b], 0));
+                if (i >= 1) CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->stream, ctx->ev_tr[b], 0));
                 if (per_launch) cudaEventRecord(ctx->ev_pool[2 * n_rec], ctx->stream);
                 launch_pair_step((const int2 *)ctx->tdesc.p, n_tiles, ctx->tlist.p, b * list_buf_entries, cap, nmp,
                                  p_np, nsg, persist_grid,
@@ -664,11 +651,18 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 if (per_launch) cudaEventRecord(ctx->ev_pool[2 * n_rec + 1], ctx->stream);
                 n_rec++;
                 ctx->launches++;
+                if (l + 2 <= maxL) {
+                    CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[b], ctx->stream));
+                    CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_st[b], 0));
+                    launch_pair_trans(djobs, nj, n_v_max, l + 2, nmp, (size_t)(b ^ 1) * list_buf_entries, l + 1,
+                                      ctx->aux);
+                    CUDA_TRY(ctx, cudaEventRecord(ctx->ev_tr[b ^ 1], ctx->aux));
+                    ctx->launches++;
+                }
                 if (l + 1 <= maxL) {
                     launch_pair_fixup(djobs, nj, n_v_max, l + 1, nmp, ctx->stream);
                     ctx->launches++;
                 }
-                CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[b], ctx->stream));
             }
             ctx->n_rec = n_rec;
         } else {

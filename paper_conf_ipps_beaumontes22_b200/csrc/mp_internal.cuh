@@ -98,7 +98,7 @@ int pair_list_cap(int max_L);
 size_t pair_entry_bytes();
 int pair_nsl(int np, int nmp);
 bool pair_supported(int P, int nmp, int n_v);
-void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int unverified_from,
+void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int fix_slab,
                        cudaStream_t s);
 void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, cudaStream_t s);
 void launch_pair_step(const int2 *tdesc, int n_tiles, const void *lists, size_t buf_off, int cap, int nmp, int np,

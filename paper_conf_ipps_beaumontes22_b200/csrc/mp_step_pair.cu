@@ -149,20 +149,15 @@ __device__ __forceinline__ int pair_vtiles(int n_v) { return (n_v + kPairVB - 1)
 // ---------------------------------------------------------------------------
 // a3 + a4 for the layer pair (l, l+1).
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l, int nmp, size_t buf_off,
-                                                         int unverified_from) {
-    // unverified_from: source slabs >= this may still be being written by the pass
-    // this launch overlaps (step(l-2) + fixup(l-1)), so their row flags are not
-    // consulted -- those entries are kept (a read of an all-+inf row is harmless)
+__device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, int l, int nmp, size_t buf_off,
+                                                int fix_slab) {
+    // fix_slab (= l-1, or -1): this launch runs concurrently with pair_fixup_kernel of
+    // slab fix_slab, which may still turn that slab's row flags on.  For a source row w
+    // of that slab whose flag is still 0, the entry is kept if the fixup could make the
+    // row finite -- its option k = fix_slab is live and reads a row of slab fix_slab-1
+    // that holds a finite value -- a superset of what the fixup will flag, so the skip
+    // stays exact.
     constexpr int KG = 32 / kPairRows;           // k values per warp iteration
-    __shared__ Job sJ;
-    if (threadIdx.x < sizeof(Job) / 8)
-        reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
-            __ldg(reinterpret_cast<const uint64_t *>(jobs + blockIdx.y) + threadIdx.x);
-    __syncthreads();
-    const Job &J = sJ;
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int vt = blockIdx.x * 4 + warp;
     if (vt >= pair_vtiles(J.n_v)) return;
     if (l > J.L) {                               // no layer l (a shorter chain of the batch):
         if (lane == 0)                           // the step kernel skips the tile
@@ -226,8 +221,17 @@ __global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l,
         for (int u = 0; u < TU; u++) {
             const int k = key[u] >> 16;
             fl[u] = 1u;
-            if (key[u] >= 0 && k - 1 < unverified_from)
-                fl[u] = J.rowflag[(size_t)(k - 1) * J.n_v + (key[u] & 0xFFFF)];
+            if (key[u] >= 0) fl[u] = J.rowflag[(size_t)(k - 1) * J.n_v + (key[u] & 0xFFFF)];
+        }
+#pragma unroll
+        for (int u = 0; u < TU; u++) {
+            const int sk = (key[u] >> 16) - 1;   // source slab
+            if (key[u] >= 0 && fl[u] == 0u && sk == fix_slab && sk >= J.kwin[sk]) {
+                const int w = key[u] & 0xFFFF;
+                int64_t d2;
+                const int32_t t2 = transition(J, sk, sk, w, __dsub_rn(J.Up[sk], J.Up[sk - 1]), &d2);
+                if (t2 >= 0 && J.rowflag[(size_t)(sk - 1) * J.n_v + (t2 & 0xFFFF)] != 0u) fl[u] = 1u;
+            }
         }
 #pragma unroll
         for (int u = 0; u < TU; u++) {
@@ -279,6 +283,16 @@ __global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l,
         if (useful) atomicAdd(J.useful, (unsigned long long)useful * per);
     }
     if (lane == 0 && n && J.segs) atomicAdd(J.segs, (unsigned long long)n);
+}
+
+__global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l, int nmp, size_t buf_off,
+                                                         int fix_slab) {
+    __shared__ Job sJ;
+    if (threadIdx.x < sizeof(Job) / 8)
+        reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
+            __ldg(reinterpret_cast<const uint64_t *>(jobs + blockIdx.y) + threadIdx.x);
+    __syncthreads();
+    pair_trans_body(sJ, blockIdx.x * 4 + (threadIdx.x >> 5), threadIdx.x & 31, l, nmp, buf_off, fix_slab);
 }
 
 // ---------------------------------------------------------------------------
@@ -623,16 +637,8 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
 // Option k = l1 of layer l1 (= l+1 of the pair): N and S from slab l1-1, which
 // the pair pass has just completed.  One warp per (job, v).
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(128) pair_fixup_kernel(const Job *jobs, int l1, int nmp) {
-    __shared__ Job sJ;
-    if (threadIdx.x < sizeof(Job) / 8)
-        reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
-            __ldg(reinterpret_cast<const uint64_t *>(jobs + blockIdx.y) + threadIdx.x);
-    __syncthreads();
-    const Job &J = sJ;
+__device__ __forceinline__ void pair_fixup_body(const Job &J, int v, int lane, int l1, int nmp) {
     if (l1 > J.L || J.P < 2) return;
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int v = blockIdx.x * 4 + warp;
     if (v >= J.n_v) return;
     const int k = l1;
     if (k < J.kwin[l1]) return;                  // U(l1,l1) > tau or its weights do not fit
@@ -655,19 +661,32 @@ __global__ void __launch_bounds__(128) pair_fixup_kernel(const Job *jobs, int l1
     const double *src = J.table + (size_t)(k - 1) * slab + (size_t)vn * rowlen;
     const double tau = J.tau;
     bool fin = false;
+    // The row already holds the clamped min of the other options (values <= tau or
+    // +inf); a cell is written back only when option k = l1 lowers it.
     for (int c = nmp + lane; c < J.P * nmp; c += 32) {       // cells p >= 1
         const int m = c & (nmp - 1);
         if (m >= J.n_m) continue;
-        double b = row[c];
+        const double b0 = row[c];
+        double b = b0;
         if (nf) b = dmin(b, src[c - nmp]);                    // N
         if ((int64_t)m + d <= (int64_t)(J.n_m - 1))           // S
             b = dmin(b, __dadd_rn(U, src[c + d]));
         b = b <= tau ? b : MP_INF;                            // clamp (Q12)
-        row[c] = b;
+        if (b < b0) row[c] = b;
         fin |= b <= tau;
     }
     if (__ballot_sync(0xffffffffu, fin) && lane == 0) atomicOr(J.rowflag + (size_t)l1 * J.n_v + v, 1u);
 }
+
+__global__ void __launch_bounds__(128) pair_fixup_kernel(const Job *jobs, int l1, int nmp) {
+    __shared__ Job sJ;
+    if (threadIdx.x < sizeof(Job) / 8)
+        reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
+            __ldg(reinterpret_cast<const uint64_t *>(jobs + blockIdx.y) + threadIdx.x);
+    __syncthreads();
+    pair_fixup_body(sJ, blockIdx.x * 4 + (threadIdx.x >> 5), threadIdx.x & 31, l1, nmp);
+}
+
 
 // tile geometry of the pair path: (v-tiles incl. kPairE extra) x p-tiles of <= 64 rows
 void pair_geom(int P, int n_v, int *np, int *n_ptiles, int *n_vtiles, int *n_tiles) {
@@ -690,10 +709,10 @@ int pair_nsl(int np, int nmp) {
 
 bool pair_supported(int P, int nmp, int n_v) { return P >= 2 && (nmp == 4 || nmp == 8) && n_v <= 65535; }
 
-void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int unverified_from,
+void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int fix_slab,
                        cudaStream_t s) {
     const int nvt = (n_v_max + kPairVB - 1) / kPairVB + kPairE;
-    pair_trans_kernel<<<dim3((nvt + 3) / 4, n_jobs), 128, 0, s>>>(jobs, l, nmp, buf_off, unverified_from);
+    pair_trans_kernel<<<dim3((nvt + 3) / 4, n_jobs), 128, 0, s>>>(jobs, l, nmp, buf_off, fix_slab);
 }
 
 void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, cudaStream_t s) {

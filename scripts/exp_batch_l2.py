@@ -21,7 +21,7 @@ while nmp < cfg["n_mem"]:
 tbytes = (cfg["L"] + 1) * cfg["n_delay"] * cfg["P"] * nmp * 8
 for B in [int(x) for x in (sys.argv[2].split(",") if len(sys.argv) > 2 else ["0", "64", "16", "8", "4", "2"])]:
     with mp.Context(0, mem_budget=(B * ((tbytes + 255) // 256 * 256) if B else 0)) as ctx:
-        ctx.set_timing(True)
+        ctx.set_timing(os.environ.get("EXP_NO_LAUNCH_TIMING") is None)
         ctx.solve_dev(dchain, *a)
         torch.cuda.synchronize()
         t0 = time.perf_counter()
