@@ -197,7 +197,10 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
     // k <= l: sources in slabs <= l-1 (final).  TU k-groups per chunk: their transitions
     // (independent global loads) and then their row flags are fetched together, so a
     // chunk costs two memory round trips instead of two per k-group.
-    constexpr int TU = 4;
+#ifndef MP_TRANS_TU
+#define MP_TRANS_TU 1
+#endif
+    constexpr int TU = MP_TRANS_TU;
     for (int kc = kA; kc <= l; kc += KG * TU) {
         int key[TU];
         uint32_t code[TU];
@@ -285,7 +288,10 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
     if (lane == 0 && n && J.segs) atomicAdd(J.segs, (unsigned long long)n);
 }
 
-__global__ void __launch_bounds__(128) pair_trans_kernel(const Job *jobs, int l, int nmp, size_t buf_off,
+#ifndef MP_TRANS_MINB
+#define MP_TRANS_MINB 1
+#endif
+__global__ void __launch_bounds__(128, MP_TRANS_MINB) pair_trans_kernel(const Job *jobs, int l, int nmp, size_t buf_off,
                                                          int fix_slab) {
     __shared__ Job sJ;
     if (threadIdx.x < sizeof(Job) / 8)
@@ -657,28 +663,45 @@ __device__ __forceinline__ void pair_fixup_body(const Job &J, int v, int lane, i
     if (!use) return;
     const size_t rowlen = (size_t)J.P * nmp;
     const size_t slab = (size_t)J.n_v * rowlen;
-    double *row = J.table + (size_t)l1 * slab + (size_t)v * rowlen;
-    const double *src = J.table + (size_t)(k - 1) * slab + (size_t)vn * rowlen;
+    double *__restrict__ row = J.table + (size_t)l1 * slab + (size_t)v * rowlen;
+    const double *__restrict__ src = J.table + (size_t)(k - 1) * slab + (size_t)vn * rowlen;
     const double tau = J.tau;
+    const int lim = J.n_m - 1 - (d > (int64_t)J.n_m ? J.n_m : (int)d);   // S valid iff m <= lim
     bool fin = false;
     // The row already holds the clamped min of the other options (values <= tau or
-    // +inf); a cell is written back only when option k = l1 lowers it.
-    for (int c = nmp + lane; c < J.P * nmp; c += 32) {       // cells p >= 1
-        const int m = c & (nmp - 1);
-        if (m >= J.n_m) continue;
-        const double b0 = row[c];
-        double b = b0;
-        if (nf) b = dmin(b, src[c - nmp]);                    // N
-        if ((int64_t)m + d <= (int64_t)(J.n_m - 1))           // S
-            b = dmin(b, __dadd_rn(U, src[c + d]));
-        b = b <= tau ? b : MP_INF;                            // clamp (Q12)
-        if (b < b0) row[c] = b;
-        fin |= b <= tau;
+    // +inf); a cell is written back only when option k = l1 lowers it.  FB cells per
+    // lane are loaded before any is stored (slab l1-1 is read-only here), so each warp
+    // keeps 3 FB loads in flight.
+    constexpr int FB = 8;
+    const int ncell = J.P * nmp;
+    for (int c0 = nmp + lane; c0 < ncell; c0 += 32 * FB) {   // cells p >= 1
+        double b0[FB], xn[FB], xs[FB];
+#pragma unroll
+        for (int i = 0; i < FB; i++) {
+            const int c = c0 + 32 * i;
+            const int m = c & (nmp - 1);
+            const bool in = c < ncell && m < J.n_m;
+            b0[i] = in ? row[c] : MP_INF;
+            xn[i] = in && nf ? __ldg(src + c - nmp) : MP_INF;          // N
+            xs[i] = in && m <= lim ? __ldg(src + c + d) : MP_INF;      // S
+        }
+#pragma unroll
+        for (int i = 0; i < FB; i++) {
+            const int c = c0 + 32 * i;
+            double b = dmin(b0[i], xn[i]);
+            if (xs[i] != MP_INF) b = dmin(b, __dadd_rn(U, xs[i]));
+            b = b <= tau ? b : MP_INF;                        // clamp (Q12)
+            if (b < b0[i]) row[c] = b;
+            fin |= b <= tau;
+        }
     }
     if (__ballot_sync(0xffffffffu, fin) && lane == 0) atomicOr(J.rowflag + (size_t)l1 * J.n_v + v, 1u);
 }
 
-__global__ void __launch_bounds__(128) pair_fixup_kernel(const Job *jobs, int l1, int nmp) {
+#ifndef MP_FIX_MINB
+#define MP_FIX_MINB 1
+#endif
+__global__ void __launch_bounds__(128, MP_FIX_MINB) pair_fixup_kernel(const Job *jobs, int l1, int nmp) {
     __shared__ Job sJ;
     if (threadIdx.x < sizeof(Job) / 8)
         reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
