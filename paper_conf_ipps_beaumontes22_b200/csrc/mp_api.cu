@@ -523,6 +523,9 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 n_v_max = std::max(n_v_max, J.n_v);
             }
             CUDA_TRY(ctx, ctx->tlist.ensure(2 * total * pair_entry_bytes()));
+            // option k = l+1 transitions of the layer-(l+1) rows: [job][2][n_v]
+            size_t voff_fx = 0;
+            CUDA_TRY(ctx, ctx->codes.ensure(2 * (size_t)nj * (size_t)disc->n_delay * sizeof(int32_t)));
             list_buf_entries = total;
             cnt_buf_entries = vtotal;
             size_t off = 0, voff = 0, ftotal = 0, wtotal = 0;
@@ -534,6 +537,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 J.tlist = (TransEntry *)((char *)ctx->tlist.p + off * pair_entry_bytes());
                 J.tcount = nullptr;
                 J.code_cap = cap;
+                J.codes = (int32_t *)ctx->codes.p + 2 * (size_t)voff_fx;
+                voff_fx += (size_t)J.n_v;
                 for (int vt = 0; vt < nvt_; vt++)
                     for (int pt = 0; pt < npt_; pt++) {
                         const size_t t = (size_t)J.tile0 + (size_t)vt * npt_ + pt;

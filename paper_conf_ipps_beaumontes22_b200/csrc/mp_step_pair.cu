@@ -190,6 +190,17 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
     const int kA = J.kwin[l];                    // window starts max(kmin_tau, kmin_W)
     const int kw = isB ? (hasB ? J.kwin[l + 1] : l + 1) : kA;
     unsigned live = 0, useful = 0;
+    // option k = l+1 of the layer-(l+1) rows, for pair_fixup_kernel: its transition
+    // (or kSkip), one word per row, buffer (pass % 2) -- the fixup of this pass runs
+    // while the next pass's lists are built
+    if (isB && row_ok && h == 0) {
+        int32_t fx = kSkip;
+        if (l + 1 >= kw) {
+            int64_t d;
+            fx = transition(J, l + 1, l + 1, v, __dsub_rn(Ul1, Ul), &d);
+        }
+        J.codes[(size_t)((l >> 1) & 1) * J.n_v + v] = fx;
+    }
     int n = 0;
     PairEntry *tl = reinterpret_cast<PairEntry *>(J.tlist) + buf_off + (size_t)vt * J.code_cap;
     PairEntry *list = tl + kPairHdr;
@@ -647,11 +658,12 @@ __device__ __forceinline__ void pair_fixup_body(const Job &J, int v, int lane, i
     if (l1 > J.L || J.P < 2) return;
     if (v >= J.n_v) return;
     const int k = l1;
-    if (k < J.kwin[l1]) return;                  // U(l1,l1) > tau or its weights do not fit
-    const double U = __dsub_rn(J.Up[l1], J.Up[l1 - 1]);
-    int64_t d;
-    const int32_t tr = transition(J, k, l1, v, U, &d);
+    // the transition of option k = l1 (pair_trans_body; kSkip if the window excludes it
+    // or neither N nor S is possible)
+    const int32_t tr = J.codes[(size_t)(((l1 - 1) >> 1) & 1) * J.n_v + v];
     if (tr < 0) return;
+    const double U = __dsub_rn(J.Up[l1], J.Up[l1 - 1]);
+    const int64_t d = (tr >> 16) & 0xFF;          // clamped to 255 (pack_trans): > n_m - 1 = no S
     const unsigned long long per = (unsigned long long)(J.P - 1) * (unsigned long long)J.n_m;
     const int vn = tr & 0xFFFF;
     const bool nf = (tr >> 24) & 1;
