@@ -337,36 +337,57 @@ static_assert(sizeof(PairMeta) == 64, "PairMeta size");
 // offset + NMP*8 + 8d.  S candidates with m + d > n_m - 1 are read (in bounds of
 // the padded ring) and discarded by predicate, so the code has no per-lane branch.
 template <int NMP>
-__device__ __forceinline__ void pair_relax(double (&best)[NMP], const char *slot, const int (&off)[NMP / 2],
+__device__ __forceinline__ void pair_relax(double (&b0)[NMP], double (&b1)[NMP], const char *slot,
+                                           const int (&off0)[NMP / 2], const int (&off1)[NMP / 2],
                                            const int (&m2)[NMP / 2], int d, bool nf, double U, int lim) {
+    // both processor rows of the thread at once: the S validity predicates (which depend
+    // on the lane's chunk rotation, not on the row) are formed once per chunk, and each
+    // is folded into the candidate's compare (one DSETP with a predicate operand and one
+    // 64-bit select per level, rather than a second select for the predicate)
     constexpr int C = NMP / 2;
     if (nf) {                                                    // N
 #pragma unroll
         for (int c = 0; c < C; c++) {
-            const double2 x = *reinterpret_cast<const double2 *>(slot + off[c]);
-            best[2 * c] = dmin(best[2 * c], x.x);
-            best[2 * c + 1] = dmin(best[2 * c + 1], x.y);
+            const double2 x = *reinterpret_cast<const double2 *>(slot + off0[c]);
+            const double2 y = *reinterpret_cast<const double2 *>(slot + off1[c]);
+            b0[2 * c] = dmin(b0[2 * c], x.x);
+            b0[2 * c + 1] = dmin(b0[2 * c + 1], x.y);
+            b1[2 * c] = dmin(b1[2 * c], y.x);
+            b1[2 * c + 1] = dmin(b1[2 * c + 1], y.y);
         }
     }
     if (lim >= 0) {                                              // S: valid iff m <= lim = n_m-1-d
         const char *srow = slot + NMP * 8 + 8 * d;
-        if ((d & 1) == 0) {
 #pragma unroll
-            for (int c = 0; c < C; c++) {
-                const double2 y = *reinterpret_cast<const double2 *>(srow + off[c]);
-                const double c0 = __dadd_rn(U, y.x), c1 = __dadd_rn(U, y.y);
-                best[2 * c] = (m2[c] <= lim && c0 < best[2 * c]) ? c0 : best[2 * c];
-                best[2 * c + 1] = (m2[c] + 1 <= lim && c1 < best[2 * c + 1]) ? c1 : best[2 * c + 1];
+        for (int c = 0; c < C; c++) {
+            const bool v0 = m2[c] <= lim, v1 = m2[c] + 1 <= lim;
+            double y0, y1, z0, z1;
+            if ((d & 1) == 0) {
+                const double2 y = *reinterpret_cast<const double2 *>(srow + off0[c]);
+                const double2 z = *reinterpret_cast<const double2 *>(srow + off1[c]);
+                y0 = y.x; y1 = y.y; z0 = z.x; z1 = z.y;
+            } else {
+                y0 = *reinterpret_cast<const double *>(srow + off0[c]);
+                y1 = *reinterpret_cast<const double *>(srow + off0[c] + 8);
+                z0 = *reinterpret_cast<const double *>(srow + off1[c]);
+                z1 = *reinterpret_cast<const double *>(srow + off1[c] + 8);
             }
-        } else {
-#pragma unroll
-            for (int c = 0; c < C; c++) {
-                const double y0 = *reinterpret_cast<const double *>(srow + off[c]);
-                const double y1 = *reinterpret_cast<const double *>(srow + off[c] + 8);
-                const double c0 = __dadd_rn(U, y0), c1 = __dadd_rn(U, y1);
-                best[2 * c] = (m2[c] <= lim && c0 < best[2 * c]) ? c0 : best[2 * c];
-                best[2 * c + 1] = (m2[c] + 1 <= lim && c1 < best[2 * c + 1]) ? c1 : best[2 * c + 1];
-            }
+            const double c0 = __dadd_rn(U, y0), c1 = __dadd_rn(U, y1);
+            const double e0 = __dadd_rn(U, z0), e1 = __dadd_rn(U, z1);
+            // b = (valid && cand < b) ? cand : b, the validity folded into the compare
+            asm("{\n\t.reg .pred q0, q1, p;\n\t"
+                "setp.ne.u32 q0, %8, 0;\n\t"
+                "setp.ne.u32 q1, %9, 0;\n\t"
+                "setp.lt.and.f64 p, %4, %0, q0;\n\t"
+                "selp.f64 %0, %4, %0, p;\n\t"
+                "setp.lt.and.f64 p, %5, %1, q1;\n\t"
+                "selp.f64 %1, %5, %1, p;\n\t"
+                "setp.lt.and.f64 p, %6, %2, q0;\n\t"
+                "selp.f64 %2, %6, %2, p;\n\t"
+                "setp.lt.and.f64 p, %7, %3, q1;\n\t"
+                "selp.f64 %3, %7, %3, p;\n\t}"
+                : "+d"(b0[2 * c]), "+d"(b0[2 * c + 1]), "+d"(b1[2 * c]), "+d"(b1[2 * c + 1])
+                : "d"(c0), "d"(c1), "d"(e0), "d"(e1), "r"((unsigned)v0), "r"((unsigned)v1));
         }
     }
 }
@@ -642,8 +663,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             const double U = isB ? M.e.U1 : M.e.U0;
             const int lim = M.n_m - 1 - d;
             const char *slot = ring + s * seg_bytes;
-            pair_relax<NMP>(b0, slot, off0, m2, d, nf, U, lim);
-            pair_relax<NMP>(b1, slot, off1, m2, d, nf, U, lim);
+            pair_relax<NMP>(b0, b1, slot, off0, off1, m2, d, nf, U, lim);
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(empty0 + 8 * s);
