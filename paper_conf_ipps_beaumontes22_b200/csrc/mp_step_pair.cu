@@ -397,15 +397,26 @@ template <int NMP>
 __device__ __forceinline__ bool pair_store(const double (&best)[NMP], double *o, int rot, double tau, int n_m) {
     constexpr int C = NMP / 2;
     bool fin = false;
+    unsigned any = 0u;
 #pragma unroll
     for (int c = 0; c < C; c++) {
         const int j = (c + rot) & (C - 1);
         double2 r;
-        r.x = (2 * j < n_m && best[2 * c] <= tau) ? best[2 * c] : MP_INF;
-        r.y = (2 * j + 1 < n_m && best[2 * c + 1] <= tau) ? best[2 * c + 1] : MP_INF;
-        fin |= (r.x <= tau) | (r.y <= tau);
+        // r = (level exists && b <= tau) ? b : +inf; any |= that predicate
+        asm("{\n\t.reg .pred q0, q1, p0, p1;\n\t"
+            "setp.lt.s32 q0, %6, %7;\n\t"
+            "setp.lt.s32 q1, %8, %7;\n\t"
+            "setp.le.and.f64 p0, %3, %5, q0;\n\t"
+            "setp.le.and.f64 p1, %4, %5, q1;\n\t"
+            "selp.f64 %0, %3, 0d7FF0000000000000, p0;\n\t"
+            "selp.f64 %1, %4, 0d7FF0000000000000, p1;\n\t"
+            "@p0 or.b32 %2, %2, 1;\n\t"
+            "@p1 or.b32 %2, %2, 1;\n\t}"
+            : "=d"(r.x), "=d"(r.y), "+r"(any)
+            : "d"(best[2 * c]), "d"(best[2 * c + 1]), "d"(tau), "r"(2 * j), "r"(n_m), "r"(2 * j + 1));
         *reinterpret_cast<double2 *>(o + 2 * j) = r;
     }
+    fin = any != 0u;
     return fin;
 }
 
