@@ -56,7 +56,7 @@ struct madpipe_ctx {
     int64_t last_load_bytes = 0, last_store_bytes = 0;   // step kernel: source segments in, rows out
     int per_launch_timing = 0;
     int kernel = -1;          // MADPIPE_KERNEL: v1 = plain loads, tma = per-tile TMA, persist, pair;
-                              // -1 (default): pair for 48 <= P <= 65 (n_mem <= 8), else persist
+                              // -1 (default): pair for P > 33 (n_mem <= 8), else persist
                               // when a row segment is >= 1 KB, else v1
     int prof = 0;             // MADPIPE_PROF=1: cycle counters of the persistent step kernel to stderr
     int n_prod = 4;           // MADPIPE_NPROD: producer warps of the persistent step kernel (1..4)
@@ -446,10 +446,11 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             int vb_, np_, npt_, nt_;
             persist_geom(cs[js[next].chain].P, disc->n_delay, nmp, &vb_, &np_, &npt_, &nt_);
             kern = (np_ + 1) * nmp * 8 >= 1024 ? 2 : 0;
-            // two-layer kernel where it measured faster (scripts/exp_dispatch.py): one
-            // processor tile that is at least 3/4 full (48 <= P <= 65), n_mem <= 8
+            // two-layer kernel where it measured faster (scripts/exp_dispatch.py,
+            // profiles/r01_pair_dispatch.md): P > 33 (the single-layer kernel needs two
+            // warps per delay row there), n_mem <= 8
             const int P = cs[js[next].chain].P;
-            if (P >= 48 && P <= 65 && pair_supported(P, nmp, disc->n_delay)) kern = 3;
+            if (P > 33 && pair_supported(P, nmp, disc->n_delay)) kern = 3;
         }
         size_t used = 0;
         int maxL = 0;

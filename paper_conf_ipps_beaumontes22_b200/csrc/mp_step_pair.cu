@@ -96,7 +96,12 @@ constexpr int kPairE = 16 / kPairVB;             // extra v-tiles: layer l+1 row
 constexpr int kPairCtas = 8 / kPairVB;           // resident CTAs per SM (one producer warp each)
 constexpr int kPairNp = 64;                      // processor rows per tile (2 per consumer thread)
 constexpr int kPairSlotsMax = 32;
-constexpr int kPairThreads = 32 * (kPairRows + 1);
+#ifndef MP_PAIR_NPROD
+#define MP_PAIR_NPROD 1
+#endif
+constexpr int kPairProd = MP_PAIR_NPROD;         // producer warps: producer p takes the CTA's tiles p, p+2, ..
+                                                 // with its own half of the ring and its own row queues
+constexpr int kPairThreads = 32 * (kPairRows + kPairProd);
 constexpr int kPairHdr = 2;                      // header entries at the head of each tile list
 #ifndef MP_POLL_NS
 #define MP_POLL_NS 100
@@ -316,7 +321,7 @@ __global__ void __launch_bounds__(128, MP_TRANS_MINB) pair_trans_kernel(const Jo
 // a5 for the layer pair: the persistent two-layer step kernel.
 // ---------------------------------------------------------------------------
 struct PairMeta {
-    int16_t flags;          // 0 = data, 1 = tile end (store the rows), 4 = terminate
+    int16_t flags;          // 0 = data, 1 = tile end (store the rows; | 16: empty tile), 4 = terminate
     int16_t np;             // processor rows of the tile
     int32_t n_m;
     union {
@@ -437,10 +442,10 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     __shared__ __align__(8) uint64_t full[kPairSlotsMax];
     __shared__ __align__(8) uint64_t empty[kPairSlotsMax];
     __shared__ __align__(16) PairMeta meta[kPairSlotsMax];
-    __shared__ uint32_t rq[kPairRows][QN];                 // per-row queues: slot | parity << 6 | code << 16
-    __shared__ int rtail[kPairRows];                       // entries pushed per row (producer)
-    __shared__ __align__(128) PairEntry stage[2][kPairStage];   // list heads of this and the next tile
-    __shared__ __align__(8) uint64_t stbar[2];
+    __shared__ uint32_t rq[kPairProd][kPairRows][QN];      // per-row queues: slot | parity << 6 | code << 16
+    __shared__ int rtail[kPairProd][kPairRows];            // entries pushed per row (producer)
+    __shared__ __align__(128) PairEntry stage[kPairProd][2][kPairStage];   // list heads of this and the next tile
+    __shared__ __align__(8) uint64_t stbar[kPairProd][2];
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
@@ -452,15 +457,19 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             mbar_init(full0 + 8 * s, 1);
             mbar_init(empty0 + 8 * s, kPairRows);
         }
-        mbar_init(smem_u32(&stbar[0]), 1);
-        mbar_init(smem_u32(&stbar[1]), 1);
+        for (int p = 0; p < kPairProd; p++) {
+            mbar_init(smem_u32(&stbar[p][0]), 1);
+            mbar_init(smem_u32(&stbar[p][1]), 1);
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    if (tid < kPairRows) rtail[tid] = 0;
+    if (tid < kPairRows * kPairProd) rtail[tid / kPairRows][tid % kPairRows] = 0;
     __syncthreads();
 
-    if (warp == kPairRows) {
-        // =========================================================== producer warp
+    if (warp >= kPairRows) {
+        // =========================================================== producer warp(s)
+        const int pw = warp - kPairRows;                   // producer index
+        const int nslp = nsl / kPairProd, s_base = pw * nslp;   // this producer's ring slots
         int sl = 0, wraps = 0;
         int tails[kPairRows];                              // entries pushed per row (same in every lane)
 #pragma unroll
@@ -474,13 +483,13 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 const bool mine = act && ((mask >> rr) & 1u);
                 const unsigned bal = __ballot_sync(0xffffffffu, mine);
                 if (mine)
-                    reinterpret_cast<volatile uint32_t *>(rq[rr])[(tails[rr] + __popc(bal & lt)) & (QN - 1)] =
+                    reinterpret_cast<volatile uint32_t *>(rq[pw][rr])[(tails[rr] + __popc(bal & lt)) & (QN - 1)] =
                         ent | (uint32_t)((codes >> (8 * rr)) & 0xFFu) << 16;
                 tails[rr] += __popc(bal);
                 if (lane == rr) mytail = tails[rr];
             }
             __syncwarp();
-            if (lane < kPairRows) st_publish(&rtail[lane], mytail);
+            if (lane < kPairRows) st_publish(&rtail[pw][lane], mytail);
         };
         // prof (MADPIPE_PROF=1): [0] producer cycles, [1] empty-barrier waits (max over lanes),
         // [2] tile setup (header), [3] consumer cycles, [4] queue waits, [5] full waits, [6] data
@@ -488,19 +497,20 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
         long long t_p0 = clock64(), t_we = 0, t_set = 0, n_tl = 0, t_push = 0;
         // the head of each tile's list (header + first entries) is bulk-copied into a
         // staging buffer one tile ahead, so a tile starts without a global-load round trip
-        const uint32_t st0 = smem_u32(&stbar[0]);
+        const uint32_t st0 = smem_u32(&stbar[pw][0]);
         const uint32_t stage_bytes = (uint32_t)stage_n * (uint32_t)sizeof(PairEntry);
         auto stage_copy = [&](int2 dsc, int buf) {
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             mbar_arrive_expect_tx(st0 + 8 * buf, stage_bytes);
-            bulk_g2s(smem_u32(&stage[buf][0]), lists + dsc.x, stage_bytes, st0 + 8 * buf);
+            bulk_g2s(smem_u32(&stage[pw][buf][0]), lists + dsc.x, stage_bytes, st0 + 8 * buf);
         };
-        const int G = (int)gridDim.x;
-        int2 desc = blockIdx.x < n_tiles ? __ldg(tdesc + blockIdx.x) : make_int2(0, 0);
-        int2 nextd = (int)blockIdx.x + G < n_tiles ? __ldg(tdesc + blockIdx.x + G) : make_int2(0, 0);
-        if (lane == 0 && (int)blockIdx.x < n_tiles) stage_copy(desc, 0);
+        const int G = (int)gridDim.x * kPairProd;           // tile stride of this producer
+        const int t0 = (int)blockIdx.x + pw * (int)gridDim.x;
+        int2 desc = t0 < n_tiles ? __ldg(tdesc + t0) : make_int2(0, 0);
+        int2 nextd = t0 + G < n_tiles ? __ldg(tdesc + t0 + G) : make_int2(0, 0);
+        if (lane == 0 && t0 < n_tiles) stage_copy(desc, 0);
         int it = 0;
-        for (int tile = blockIdx.x; tile < n_tiles; tile += G, it++) {
+        for (int tile = t0; tile < n_tiles; tile += G, it++) {
             const long long t_t0 = prof ? clock64() : 0;
             const int buf = it & 1;
             if (lane == 0 && tile + G < n_tiles) stage_copy(nextd, buf ^ 1);
@@ -509,21 +519,23 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             nextd = tile + 2 * G < n_tiles ? __ldg(tdesc + tile + 2 * G) : make_int2(0, 0);
             mbar_wait(st0 + 8 * buf, (uint32_t)((it >> 1) & 1));
             const PairEntry *tl = lists + mine.x;
-            const PairEntry *sg = stage[buf];
+            const PairEntry *sg = stage[pw][buf];
             const PairHdr hd = *reinterpret_cast<const PairHdr *>(sg);
-            if (hd.n < 0) continue;                       // the job has no layer l
             auto entry = [&](int e) -> PairEntry { return e + kPairHdr < stage_n ? sg[kPairHdr + e] : tl[kPairHdr + e]; };
-            // first round's entries
-            PairEntry cur;
-            if (lane < round) cur = entry(lane);
             const int pt = mine.y;
             const int p_lo = 1 + pt * np_max;
             const int np = min(np_max, hd.P - p_lo);
-            if (np <= 0) continue;
+            // a job with no layer l, or no processors in this tile: no entries and an empty
+            // tile end (consumers keep one tile end per tile: with two producers they take
+            // the tiles' ends in turn)
+            const bool skip = hd.n < 0 || np <= 0;
+            // first round's entries
+            PairEntry cur;
+            if (!skip && lane < round) cur = entry(lane);
             const int64_t rowlen = (int64_t)hd.P * NMP;
             const int64_t slab = (int64_t)hd.n_v * rowlen;
             const uint32_t seg_bytes = (uint32_t)(np + 1) * NMP * 8u;
-            const int n = hd.n;
+            const int n = skip ? 0 : hd.n;
             const int stages = n + 1;                      // entries, then the tile-end marker
             if (prof) { t_set += clock64() - t_t0; n_tl++; }
             for (int r0 = 0; r0 < stages; r0 += round) {
@@ -535,7 +547,8 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 uint64_t codes = 0;                         // in a register (an array was spilled)
                 if (act) {
                     int s = sl + lane, use = wraps;
-                    if (s >= nsl) { s -= nsl; use++; }
+                    if (s >= nslp) { s -= nslp; use++; }
+                    s += s_base;
                     const long long tw = prof ? clock64() : 0;
                     if (use > 0) mbar_wait(empty0 + 8 * s, (uint32_t)((use - 1) & 1));
                     if (prof) {
@@ -563,7 +576,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                         mbar_arrive_expect_tx(full0 + 8 * s, seg_bytes);
                     } else {
                         mask = (1u << kPairRows) - 1u;
-                        M.flags = 1;
+                        M.flags = skip ? (1 | 16) : 1;
                         M.t.tau = hd.tau;
                         M.t.flA = hd.flA;
                         M.slab = slab;
@@ -582,17 +595,18 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 cur = nxt;
                 const int adv = min(round, stages - r0);
                 sl += adv;
-                if (sl >= nsl) { sl -= nsl; wraps++; }
+                if (sl >= nslp) { sl -= nslp; wraps++; }
             }
         }
         {                                                  // terminate every row
             const bool act = lane == 0;
             uint32_t ent = 0;
             if (act) {
-                if (wraps > 0) mbar_wait(empty0 + 8 * sl, (uint32_t)((wraps - 1) & 1));
-                meta[sl].flags = 4;
-                ent = (uint32_t)sl | (uint32_t)(wraps & 1) << 6;
-                mbar_arrive(full0 + 8 * sl);
+                const int sg_ = s_base + sl;
+                if (wraps > 0) mbar_wait(empty0 + 8 * sg_, (uint32_t)((wraps - 1) & 1));
+                meta[sg_].flags = 4;
+                ent = (uint32_t)sg_ | (uint32_t)(wraps & 1) << 6;
+                mbar_arrive(full0 + 8 * sg_);
             }
             push(act, (1u << kPairRows) - 1u, ent, 0ull);
         }
@@ -624,19 +638,20 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     for (int i = 0; i < NMP; i++) { b0[i] = MP_INF; b1[i] = MP_INF; }
     const char *ring = reinterpret_cast<const char *>(dsm);
     const int seg_bytes = seg_doubles * 8;
-    int head = 0;
+    int head[kPairProd] = {};
+    int qp = 0;                                            // the queue of the current tile's producer
     long long t_c0 = clock64(), t_q = 0, t_f = 0, n_sl = 0;
     for (;;) {
         const long long ta = prof ? clock64() : 0;
         // an empty queue: back off instead of spinning (a spinning warp takes issue slots
         // from the producer and the working rows)
-        while (ld_poll(&rtail[r]) == head) {
+        while (ld_poll(&rtail[qp][r]) == head[qp]) {
 #if MP_POLL_NS > 0
             __nanosleep(MP_POLL_NS);
 #endif
         }
-        const uint32_t ent = reinterpret_cast<volatile uint32_t *>(rq[r])[head & (QN - 1)];
-        head++;
+        const uint32_t ent = reinterpret_cast<volatile uint32_t *>(rq[qp][r])[head[qp] & (QN - 1)];
+        head[qp]++;
         const int s = (int)(ent & 63u);                    // this row's slot
         const long long tb = prof ? clock64() : 0;
         mbar_wait(full0 + 8 * s, (ent >> 6) & 1u);
@@ -655,7 +670,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
         if (flags & 1) {                                   // tile end: clamp (Q12), store, flag
             const int np = M.np, n_m = M.n_m;
             const int v = isB ? M.t.v0B + (r - kPairVB) : M.t.v0A + r;
-            const bool ok = (!isB || M.hasB) && v >= 0 && v < M.n_v;
+            const bool ok = !(flags & 16) && (!isB || M.hasB) && v >= 0 && v < M.n_v;   // 16: empty tile
             bool fin = false;
             if (ok) {
                 double *o = M.t.outA + (int64_t)(v - M.t.v0A) * M.rowlen + (isB ? M.slab : (int64_t)0);
@@ -666,6 +681,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 atomicOr(M.t.flA + (isB ? M.n_v : 0) + v, 1u);
 #pragma unroll
             for (int i = 0; i < NMP; i++) { b0[i] = MP_INF; b1[i] = MP_INF; }
+            if (kPairProd > 1) qp = (qp + 1) % kPairProd;   // the next tile comes from the next producer
         } else {
             // rows lane and lane+32 are relaxed whether or not they exist in this tile
             // (np < 64): the extra rows read in-bounds ring bytes and are never stored
@@ -770,7 +786,8 @@ size_t pair_entry_bytes() { return sizeof(PairEntry); }
 int pair_nsl(int np, int nmp) {
     const int seg = (np + 1) * nmp * 8;
     int slots = (200 * 1024 / kPairCtas) / seg;
-    return slots > kPairSlotsMax ? kPairSlotsMax : slots;
+    slots = slots > kPairSlotsMax ? kPairSlotsMax : slots;
+    return slots - slots % kPairProd;                       // split evenly between the producers
 }
 
 bool pair_supported(int P, int nmp, int n_v) { return P >= 2 && (nmp == 4 || nmp == 8) && n_v <= 65535; }
@@ -807,7 +824,7 @@ void launch_pair_step(const int2 *tdesc, int n_tiles, const void *lists, size_t 
 #define MP_CASE(N)                                                                                     \
     case N:                                                                                            \
         cudaFuncSetAttribute(pair_step_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);   \
-        pair_step_kernel<N><<<grid, kPairThreads, smem, s>>>(tdesc, n_tiles, L, np, nsl, pair_round(nsl), stage_n, prof); \
+        pair_step_kernel<N><<<grid, kPairThreads, smem, s>>>(tdesc, n_tiles, L, np, nsl, pair_round(nsl / kPairProd), stage_n, prof); \
         break;
         MP_CASE(4) MP_CASE(8)
 #undef MP_CASE
