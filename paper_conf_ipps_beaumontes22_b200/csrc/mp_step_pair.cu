@@ -442,7 +442,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     __shared__ __align__(8) uint64_t full[kPairSlotsMax];
     __shared__ __align__(8) uint64_t empty[kPairSlotsMax];
     __shared__ __align__(16) PairMeta meta[kPairSlotsMax];
-    __shared__ uint32_t rq[kPairProd][kPairRows][QN];      // per-row queues: slot | parity << 6 | code << 16
+    __shared__ uint32_t rq[kPairProd][kPairRows][QN];      // per-row queues: slot | parity << 6 | n_m << 8 | code << 16
     __shared__ int rtail[kPairProd][kPairRows];            // entries pushed per row (producer)
     __shared__ __align__(128) PairEntry stage[kPairProd][2][kPairStage];   // list heads of this and the next tile
     __shared__ __align__(8) uint64_t stbar[kPairProd][2];
@@ -556,10 +556,9 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                         const unsigned mx = __reduce_max_sync(__activemask(), dw);
                         if (lane == 0) t_we += mx;
                     }
-                    ent = (uint32_t)s | (uint32_t)(use & 1) << 6;
+                    // queue entry: slot | parity << 6 | n_m << 8 | row code << 16 (n_m <= 8)
+                    ent = (uint32_t)s | (uint32_t)(use & 1) << 6 | (uint32_t)hd.n_m << 8;
                     PairMeta &M = meta[s];
-                    M.np = (int16_t)np;
-                    M.n_m = hd.n_m;
                     if (q < n) {
                         bulk_g2s(ring_s + 8u * (uint32_t)(s * seg_doubles),
                                  hd.table + (int64_t)(cur.k - 1) * slab + (int64_t)cur.vp * rowlen +
@@ -576,6 +575,8 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                         mbar_arrive_expect_tx(full0 + 8 * s, seg_bytes);
                     } else {
                         mask = (1u << kPairRows) - 1u;
+                        M.np = (int16_t)np;
+                        M.n_m = hd.n_m;
                         M.flags = skip ? (1 | 16) : 1;
                         M.t.tau = hd.tau;
                         M.t.flA = hd.flA;
@@ -638,17 +639,22 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     for (int i = 0; i < NMP; i++) { b0[i] = MP_INF; b1[i] = MP_INF; }
     const char *ring = reinterpret_cast<const char *>(dsm);
     const int seg_bytes = seg_doubles * 8;
-    int head[kPairProd] = {};
+    int head[kPairProd] = {}, avail[kPairProd] = {};
     int qp = 0;                                            // the queue of the current tile's producer
     long long t_c0 = clock64(), t_q = 0, t_f = 0, n_sl = 0;
     for (;;) {
         const long long ta = prof ? clock64() : 0;
         // an empty queue: back off instead of spinning (a spinning warp takes issue slots
         // from the producer and the working rows)
-        while (ld_poll(&rtail[qp][r]) == head[qp]) {
+        // (the tail is re-read only when the entries seen last time are used up)
+        if (head[qp] == avail[qp]) {
+            int t;
+            while ((t = ld_poll(&rtail[qp][r])) == head[qp]) {
 #if MP_POLL_NS > 0
-            __nanosleep(MP_POLL_NS);
+                __nanosleep(MP_POLL_NS);
 #endif
+            }
+            avail[qp] = t;
         }
         const uint32_t ent = reinterpret_cast<volatile uint32_t *>(rq[qp][r])[head[qp] & (QN - 1)];
         head[qp]++;
@@ -688,7 +694,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             const int d = (int)((ent >> 16) & 127u);
             const bool nf = (ent >> 23) & 1u;
             const double U = isB ? M.e.U1 : M.e.U0;
-            const int lim = M.n_m - 1 - d;
+            const int lim = (int)((ent >> 8) & 15u) - 1 - d;   // n_m - 1 - d
             const char *slot = ring + s * seg_bytes;
             pair_relax<NMP>(b0, b1, slot, off0, off1, m2, d, nf, U, lim);
         }
