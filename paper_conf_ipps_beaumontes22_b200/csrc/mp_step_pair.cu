@@ -442,7 +442,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     __shared__ __align__(8) uint64_t full[kPairSlotsMax];
     __shared__ __align__(8) uint64_t empty[kPairSlotsMax];
     __shared__ __align__(16) PairMeta meta[kPairSlotsMax];
-    __shared__ uint32_t rq[kPairProd][kPairRows][QN];      // per-row queues: slot | parity << 6 | n_m << 8 | code << 16
+    __shared__ uint32_t rq[kPairProd][kPairRows][QN];      // per-row queues: slot | parity << 6 | control << 7 | n_m << 8 | code << 16
     __shared__ int rtail[kPairProd][kPairRows];            // entries pushed per row (producer)
     __shared__ __align__(128) PairEntry stage[kPairProd][2][kPairStage];   // list heads of this and the next tile
     __shared__ __align__(8) uint64_t stbar[kPairProd][2];
@@ -556,7 +556,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                         const unsigned mx = __reduce_max_sync(__activemask(), dw);
                         if (lane == 0) t_we += mx;
                     }
-                    // queue entry: slot | parity << 6 | n_m << 8 | row code << 16 (n_m <= 8)
+                    // queue entry: slot | parity << 6 | control << 7 | n_m << 8 | row code << 16 (n_m <= 8)
                     ent = (uint32_t)s | (uint32_t)(use & 1) << 6 | (uint32_t)hd.n_m << 8;
                     PairMeta &M = meta[s];
                     if (q < n) {
@@ -565,7 +565,6 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                                      (int64_t)(p_lo - 1) * NMP,
                                  seg_bytes, full0 + 8 * s);
                         mask = cur.mask;
-                        M.flags = 0;
                         M.e.U0 = cur.U0;
                         M.e.U1 = cur.U1;
                         static_assert(kPairRows <= 8, "codes packing");
@@ -575,6 +574,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                         mbar_arrive_expect_tx(full0 + 8 * s, seg_bytes);
                     } else {
                         mask = (1u << kPairRows) - 1u;
+                        ent |= 128u;                       // control slot
                         M.np = (int16_t)np;
                         M.n_m = hd.n_m;
                         M.flags = skip ? (1 | 16) : 1;
@@ -606,7 +606,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 const int sg_ = s_base + sl;
                 if (wraps > 0) mbar_wait(empty0 + 8 * sg_, (uint32_t)((wraps - 1) & 1));
                 meta[sg_].flags = 4;
-                ent = (uint32_t)sg_ | (uint32_t)(wraps & 1) << 6;
+                ent = (uint32_t)sg_ | (uint32_t)(wraps & 1) << 6 | 128u;   // control slot
                 mbar_arrive(full0 + 8 * sg_);
             }
             push(act, (1u << kPairRows) - 1u, ent, 0ull);
@@ -663,6 +663,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
         mbar_wait(full0 + 8 * s, (ent >> 6) & 1u);
         if (prof) { const long long tc = clock64(); t_q += tb - ta; t_f += tc - tb; n_sl++; }
         const PairMeta &M = meta[s];
+        if (ent & 128u) {                                  // control slot (tile end / terminate)
         const int flags = M.flags;
         if (flags & 4) {
             if (prof && lane == 0) {
@@ -688,6 +689,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
 #pragma unroll
             for (int i = 0; i < NMP; i++) { b0[i] = MP_INF; b1[i] = MP_INF; }
             if (kPairProd > 1) qp = (qp + 1) % kPairProd;   // the next tile comes from the next producer
+        }
         } else {
             // rows lane and lane+32 are relaxed whether or not they exist in this tile
             // (np < 64): the extra rows read in-bounds ring bytes and are never stored
