@@ -310,3 +310,29 @@ def test_batch_mixed_lengths(kernel):
     for ch, M, got in zip(chains, Ms, res):
         ref = oracle.solve(ch, P, M, 30.0, n_m, n_v, n_c, v_range=1, n_threads=4)
         _same_solution(got, ref)
+
+
+def test_work_counters_agree_across_kernels():
+    """The live-relaxation counter (madpipe_last_counts: effective_updates) is a property
+    of the DP instance, not of the kernel: the two-layer path (counted by its trans and
+    fixup kernels) must report the same count as the one-layer kernels.  The useful count
+    (live and reading a finite source row) is kept by the persistent kernels only and is
+    bounded by the effective count."""
+    rng = np.random.default_rng(21)
+    ch = chaingen.tiny(rng, 20)
+    P, n_m, n_v, n_c = 48, 8, 96, 5
+    M = int((3 * ch["W"].sum() + 3 * ch["a"].sum()) * 0.5) + 1
+    counts = {}
+    for kernel in ("pair", "persist", "v1"):
+        c = _ctx_with_kernel(kernel)
+        try:
+            c.solve(ch, P, M, 30.0, n_m, n_v, n_c, v_range=1)
+            counts[kernel] = c.last_counts()
+        finally:
+            c.close()
+    for kernel, got in counts.items():
+        assert got["cell_updates"] == counts["v1"]["cell_updates"], kernel
+        assert got["effective_updates"] == counts["v1"]["effective_updates"], (kernel, counts)
+        assert got["useful_updates"] <= got["effective_updates"], (kernel, got)
+        if kernel != "v1":
+            assert got["useful_updates"] > 0, (kernel, got)
