@@ -106,6 +106,9 @@ constexpr int kPairHdr = 2;                      // header entries at the head o
 #ifndef MP_POLL_NS
 #define MP_POLL_NS 100
 #endif
+#ifndef MP_PAIR_PROF
+#define MP_PAIR_PROF 1                                     // MADPIPE_PROF=1 cycle counters in pair_step_kernel
+#endif
 #ifndef MP_PAIR_STAGE
 #define MP_PAIR_STAGE 32
 #endif
@@ -436,6 +439,9 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     // count) releases the slot's empty barrier.  Tile ends and the final
     // termination are slots without data pushed to all rows.  tdesc[tile] =
     // (offset of the tile's list in `lists`, processor tile).
+#if !MP_PAIR_PROF
+    prof = nullptr;                                        // cycle counters compiled out (MADPIPE_PROF reads zeros)
+#endif
     constexpr int C = NMP / 2;
     constexpr int QN = 32;                                 // queue entries per row (>= slots)
     extern __shared__ __align__(128) unsigned char dsm[];
@@ -739,7 +745,10 @@ __device__ __forceinline__ void pair_fixup_body(const Job &J, int v, int lane, i
     // +inf); a cell is written back only when option k = l1 lowers it.  FB cells per
     // lane are loaded before any is stored (slab l1-1 is read-only here), so each warp
     // keeps 3 FB loads in flight.
-    constexpr int FB = 8;
+#ifndef MP_FIX_FB
+#define MP_FIX_FB 8
+#endif
+    constexpr int FB = MP_FIX_FB;
     const int ncell = J.P * nmp;
     for (int c0 = nmp + lane; c0 < ncell; c0 += 32 * FB) {   // cells p >= 1
         double b0[FB], xn[FB], xs[FB];
