@@ -104,7 +104,7 @@ constexpr int kPairProd = MP_PAIR_NPROD;         // producer warps: producer p t
 constexpr int kPairThreads = 32 * (kPairRows + kPairProd);
 constexpr int kPairHdr = 2;                      // header entries at the head of each tile list
 #ifndef MP_POLL_NS
-#define MP_POLL_NS 100
+#define MP_POLL_NS 250
 #endif
 #ifndef MP_PAIR_PROF
 #define MP_PAIR_PROF 1                                     // MADPIPE_PROF=1 cycle counters in pair_step_kernel
@@ -746,7 +746,7 @@ __device__ __forceinline__ void pair_fixup_body(const Job &J, int v, int lane, i
     // lane are loaded before any is stored (slab l1-1 is read-only here), so each warp
     // keeps 3 FB loads in flight.
 #ifndef MP_FIX_FB
-#define MP_FIX_FB 8
+#define MP_FIX_FB 4
 #endif
     constexpr int FB = MP_FIX_FB;
     const int ncell = J.P * nmp;
