@@ -308,7 +308,7 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
 }
 
 #ifndef MP_TRANS_MINB
-#define MP_TRANS_MINB 1
+#define MP_TRANS_MINB 8
 #endif
 __global__ void __launch_bounds__(128, MP_TRANS_MINB) pair_trans_kernel(const Job *jobs, int l, int nmp, size_t buf_off,
                                                          int fix_slab) {
