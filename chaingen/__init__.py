@@ -232,8 +232,10 @@ def toy(seed: int = 1, L: int = 8):
 
 
 def tiny(rng: np.random.Generator, L: int, integer_times: bool = False, mem_scale: float = 1.0,
-         zero_mem: bool = False):
-    """Small random chain for fuzz tests (brute force sizes)."""
+         zero_mem: bool = False, a_hi: int = 40):
+    """Small random chain for fuzz tests (brute force sizes).  ``a_hi`` bounds the
+    activation sizes (exclusive); a large value with a small beta gives
+    communication-bound chains (C(i) = 2 a_i / beta above the period)."""
     if integer_times:
         uF = rng.integers(1, 6, size=L).astype(np.float64)
         uB = rng.integers(1, 11, size=L).astype(np.float64)
@@ -244,7 +246,7 @@ def tiny(rng: np.random.Generator, L: int, integer_times: bool = False, mem_scal
         W = np.zeros(L, np.int64); a = np.zeros(L + 1, np.int64)
     else:
         W = (rng.integers(1, 20, size=L) * mem_scale).astype(np.int64)
-        a = (rng.integers(1, 40, size=L + 1) * mem_scale).astype(np.int64)
+        a = (rng.integers(1, a_hi, size=L + 1) * mem_scale).astype(np.int64)
     return _finish("tiny%d" % L, uF, uB, W, a)
 
 

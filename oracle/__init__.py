@@ -31,7 +31,9 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "madpipe_oracle.c")
-_LIB = os.path.join(_HERE, "liboracle.so")
+# ORACLE_LIB: a prebuilt alternative (only scripts/mutate_oracle.py uses it, to run the
+# pins against deliberately broken copies of madpipe_oracle.c)
+_LIB = os.environ.get("ORACLE_LIB") or os.path.join(_HERE, "liboracle.so")
 _lock = threading.Lock()
 _lib = None
 
@@ -44,6 +46,8 @@ INFEASIBLE = 1
 
 def build(force: bool = False) -> str:
     """Compile liboracle.so (plain C, no FMA contraction, OpenMP over candidates)."""
+    if os.environ.get("ORACLE_LIB"):
+        return _LIB
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + ".tmp.%d" % os.getpid()
         cmd = ["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math", "-fopenmp",

@@ -73,3 +73,19 @@ def test_algorithm1_invariants():
         alloc = [((f, l), 1 if pr == P - 1 else 0) for (f, l, pr) in r["stages"]]
         val = bruteforce.literal_evaluate(c, r["That"][i], n_t, alloc, P - 1, 0, 0, 0)
         assert val == r["T"][i]
+
+
+def test_golden_algorithm1_four_iterations():
+    """Hand-worked Algorithm 1 (tests/golden, 'algorithm1_four_iterations'): the That_i
+    sequence follows reading Q15; the printed order of P:205 would diverge at i = 2."""
+    import json
+    import os
+    g = os.path.join(os.path.dirname(__file__), "golden", "hand_worked.json")
+    ex = json.load(open(g))["examples"][3]
+    beta = math.inf if ex["beta"] == "inf" else float(ex["beta"])
+    r = oracle.literal_solve(ex["chain"], ex["P"], ex["M"], beta, ex["n_m"], ex["n_v"], ex["n_t"], K=ex["K"])
+    e = ex["expect"]
+    assert list(r["That"]) == e["That"]
+    assert list(r["T"]) == e["T"]
+    assert r["period"] == e["period"] and r["best_iter"] == e["best_iter"]
+    assert [list(s) for s in r["stages"]] == e["stages"]

@@ -360,3 +360,129 @@ def test_table_monotone_in_processors():
                 if col.any():
                     first = int(np.argmax(col))
                     assert col[first:].all()
+
+
+# ------------------------------------------------------------------ communication-bound chains
+def _rand_comm_case(rng, L=None, P=None):
+    """A family where boundaries are expensive: activations up to 400 bytes with
+    beta in [5, 30] (C(i) = 2 a_i / beta up to 160 s against stage loads of a few
+    seconds), so C(k-1) > tau prunes splits and a link is often the
+    bottleneck of the allocation period."""
+    L = int(rng.integers(2, 7)) if L is None else L
+    P = int(rng.integers(1, 4)) if P is None else P
+    ch = chaingen.tiny(rng, L, a_hi=400)
+    n_m = int(rng.choice([2, 4, 8]))
+    n_v = int(rng.choice([4, 8, 16]))
+    v_range = int(rng.integers(0, 2))
+    total_mem = 3 * int(np.sum(ch["W"])) + 3 * int(np.sum(ch["a"]))
+    M = int(total_mem * rng.uniform(0.15, 0.9)) + 1
+    beta = float(rng.uniform(5.0, 30.0))
+    return ch, P, M, beta, n_m, n_v, v_range
+
+
+def _comm_taus(pre):
+    """Periods around the loads, where the comm constraint bites: lb, 1.5 lb, 2.5 lb,
+    a tenth of the way to ub, and U(1,L)."""
+    lb, ub = pre["lb"], pre["ub"]
+    return (lb, 1.5 * lb, 2.5 * lb, lb + 0.1 * (ub - lb), pre["Up"][-1])
+
+
+def test_root_equals_bruteforce_comm_heavy():
+    """[S3] on the communication-bound family: the DP root equals the brute-force
+    minimum bit for bit, and the family really exercises C(k-1) > tau."""
+    rng = np.random.default_rng(25)
+    total = with_c = n_fin = 0
+    for _ in range(150):
+        ch, P, M, beta, n_m, n_v, vr = _rand_comm_case(rng)
+        pre = oracle.prep(ch, P, beta)
+        L = len(ch["uF"])
+        cmax = max(pre["C"][1:L])
+        for tau in _comm_taus(pre):
+            A, _, _ = oracle.table(ch, P, M, beta, n_m, n_v, vr, tau, with_arg=False)
+            bf, _ = bruteforce.root(ch, P, M, beta, n_m, n_v, vr, tau)
+            dp = A[-1, P - 1, 0, 0]
+            assert dp == bf, (ch, P, M, beta, n_m, n_v, vr, tau, dp, bf)
+            total += 1
+            with_c += cmax > tau
+            n_fin += dp < INF
+    assert with_c >= 0.3 * total and n_fin >= 0.3 * total, (with_c, n_fin, total)
+
+
+def test_comm_constraint_binds():
+    """The C(k-1) <= tau rule changes the answer on this family: with the links made
+    free (beta = inf) the same chains are feasible at strictly more of these periods,
+    so a DP that ignored the rule would disagree with the brute force above."""
+    rng = np.random.default_rng(26)
+    differ = 0
+    for _ in range(100):
+        ch, P, M, beta, n_m, n_v, vr = _rand_comm_case(rng)
+        pre = oracle.prep(ch, P, beta)
+        for tau in _comm_taus(pre):
+            A, _, _ = oracle.table(ch, P, M, beta, n_m, n_v, vr, tau, with_arg=False)
+            bf_free, _ = bruteforce.root(ch, P, M, math.inf, n_m, n_v, vr, tau)
+            differ += (A[-1, P - 1, 0, 0] == INF) and bf_free < INF
+    assert differ >= 20, differ
+
+
+def test_every_cell_equals_bruteforce_comm_heavy():
+    rng = np.random.default_rng(27)
+    for _ in range(16):
+        ch, P, M, beta, n_m, n_v, vr = _rand_comm_case(rng, L=int(rng.integers(2, 5)),
+                                                        P=int(rng.integers(1, 4)))
+        n_v = 4
+        n_m = int(rng.choice([2, 4]))
+        pre = oracle.prep(ch, P, beta)
+        tau = 1.5 * pre["lb"]
+        A, _, _ = oracle.table(ch, P, M, beta, n_m, n_v, vr, tau)
+        L = len(ch["uF"])
+        for l in range(L + 1):
+            for p in range(P):
+                for v in range(n_v):
+                    for m in range(n_m):
+                        bf = bruteforce.cell(ch, P, M, beta, n_m, n_v, vr, tau, l, p, v, m)
+                        assert A[l, p, v, m] == bf, (l, p, v, m)
+
+
+def test_traceback_verified_comm_heavy():
+    """[S4] on the communication-bound family, with a grid that starts near lb: the
+    simulator recomputes the allocation period including every link, so a
+    load_period that missed the link term, or an allocation with a link above tau,
+    fails here."""
+    rng = np.random.default_rng(28)
+    checked = link_bound = 0
+    for _ in range(200):
+        ch, P, M, beta, n_m, n_v, vr = _rand_comm_case(rng, L=int(rng.integers(3, 8)))
+        r = oracle.solve(ch, P, M, beta, n_m, n_v, n_c=400, v_range=vr)
+        if r["rc"] != 0:
+            continue
+        val = bruteforce.value_of_stages(ch, P, M, beta, n_m, n_v, vr, r["period"], r["stages"])
+        assert val == r["special_load"] == r["root"][r["cand_index"]]
+        rep = simulator.check_allocation(ch, P, M, beta, r["period"], r["stages"],
+                                         r["load_period"], r["special_load"], build_pattern=False)
+        assert rep["errors"] == [], rep["errors"]
+        loads = [sum(ch["uF"][i] + ch["uB"][i] for i in range(k - 1, l)) for (k, l, p) in r["stages"]
+                 if p != P - 1]
+        links = [2.0 * ch["a"][k - 1] / beta for (k, l, p) in r["stages"] if k > 1]
+        link_bound += bool(links) and max(links) > max(loads + [r["special_load"]])
+        checked += 1
+    assert checked > 100 and link_bound >= 10, (checked, link_bound)
+
+
+def test_golden_communication_forces_merge():
+    ex = json.load(open(GOLD))["examples"][2]
+    r = oracle.solve(ex["chain"], ex["P"], ex["M"], _beta(ex["beta"]), ex["n_m"], ex["n_v"],
+                     ex["n_c"], v_range=ex["v_range"])
+    e = ex["expect"]
+    assert list(r["tau"][:3]) == e["tau_first"]
+    assert r["root"][0] == INF
+    assert r["cand_index"] == e["cand_index"]
+    assert r["period"] == e["period"] and r["special_load"] == e["special_load"]
+    assert r["load_period"] == e["load_period"]
+    assert [list(s) for s in r["stages"]] == e["stages"]
+
+
+def test_golden_tau_grid_rounding():
+    ex = json.load(open(GOLD))["examples"][4]
+    r = oracle.solve(ex["chain"], ex["P"], ex["M"], _beta(ex["beta"]), ex["n_m"], ex["n_v"],
+                     ex["n_c"], v_range=ex["v_range"])
+    assert [float.fromhex(h) for h in ex["expect"]["tau_hex"]] == list(r["tau"])
