@@ -40,6 +40,8 @@ extern "C" {
 #define MADPIPE_EINVAL    (-1)   /* invalid argument (see madpipe_validate)            */
 #define MADPIPE_ENOMEM    (-2)   /* device or host allocation failed                    */
 #define MADPIPE_ECUDA     (-3)   /* CUDA runtime error (no device, launch failure, ...) */
+#define MADPIPE_ENCCL     (-4)   /* NCCL unavailable (libnccl.so.2 not loadable) or an NCCL
+                                    call failed; the ctx's communicator is then unusable     */
 #define MADPIPE_ESTATE    (-5)   /* call out of order (e.g. resolve of an infeasible j) */
 
 /* A linear (or linearised) chain of L layers (section 3).
@@ -97,14 +99,30 @@ typedef struct {
 typedef struct madpipe_ctx madpipe_ctx;
 
 /* ---- context --------------------------------------------------------------
- * Create a ctx on CUDA device `device`.  `cuda_stream` is a cudaStream_t to
- * issue work on (e.g. torch.cuda.current_stream().cuda_stream), or NULL for a
- * stream owned by the ctx.  `mem_budget` bounds the device bytes used for DP
- * tables (0 = 60% of the free memory at creation).  Returns MADPIPE_ECUDA if
- * no device is usable. */
-int  madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stream, int64_t mem_budget);
+ * One process per GPU.  A ctx is bound to CUDA
+ * device `device` and is rank `rank` of `world` ranks.  With world > 1 the ctx
+ * owns an NCCL communicator built from `nccl_id` (128 bytes from
+ * madpipe_get_unique_id on one rank, distributed by the caller -- process
+ * bootstrap only), over which madpipe_solve / _solve_dev / _solve_batch run
+ * the path's single exchange step a7 (the MIN all-reduce of the candidate
+ * indices) themselves: an N-GPU solve is one call per rank, every rank passes
+ * identical inputs and receives the identical result.  With world = 1,
+ * `nccl_id` may be NULL (no communicator) or a valid id (a communicator of one
+ * rank: the same collective code path, e.g. for tests on one GPU).
+ * `cuda_stream` is a cudaStream_t to issue work on (e.g.
+ * torch.cuda.current_stream().cuda_stream), or NULL for a stream owned by the
+ * ctx.  `mem_budget` bounds the device bytes used for DP tables (0 = 60% of the
+ * free memory at creation).  Errors: MADPIPE_EINVAL (rank/world/device),
+ * MADPIPE_ECUDA (no usable device), MADPIPE_ENCCL (NCCL missing or
+ * ncclCommInitRank failed).  NCCL is loaded at run time (dlopen of
+ * libnccl.so.2, or MADPIPE_NCCL_LIB). */
+int  madpipe_get_unique_id(uint8_t id[128]);
+int  madpipe_ctx_create(madpipe_ctx **out, int device, int32_t rank, int32_t world,
+                        const uint8_t *nccl_id, void *cuda_stream, int64_t mem_budget);
 void madpipe_ctx_destroy(madpipe_ctx *ctx);
 const char *madpipe_last_error(const madpipe_ctx *ctx);   /* ctx may be NULL */
+/* rank, world and the loaded NCCL version (0 = no communicator); any may be NULL. */
+int  madpipe_ctx_info(const madpipe_ctx *ctx, int32_t *rank, int32_t *world, int32_t *nccl_version);
 
 /* ---- host-only helpers (no GPU needed) ------------------------------------ */
 /* Check every argument rule of this header; MADPIPE_OK or MADPIPE_EINVAL.
@@ -124,24 +142,29 @@ int64_t madpipe_cell_updates(const madpipe_chain *chain, int32_t P, const madpip
                              double tau);
 
 /* ---- the hot path -----------------------------------------------------------
- * Full solve on one GPU (world = 1): profile prep (a1), candidate grid (a2),
- * the batched wavefront DP over every candidate (a3-a5), root test and
- * minimum (a6), winner re-solve and device traceback (a8), result (a9).
- * [host] chain and output. */
+ * Full solve: profile prep (a1), candidate grid (a2), the batched wavefront DP
+ * over this rank's candidates (a3-a5; rank r of W owns j = r, r+W, ..., as
+ * madpipe_shard), root test and local minimum (a6), the MIN all-reduce of the
+ * ranks' smallest feasible index over the ctx's communicator (a7; skipped
+ * without one), winner re-solve and device traceback on every rank (a8),
+ * result (a9).  With disc->early_exit = 2 each of the two rounds (coarse, then
+ * the gap) is split over the ranks and ends in one all-reduce.
+ * out->cell_updates counts this rank's relaxations.  [host] chain and output. */
 int madpipe_solve(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
                   double beta, const madpipe_disc *disc, madpipe_alloc *out);
 /* Same, with the chain arrays already resident in device memory ([dev]). */
 int madpipe_solve_dev(madpipe_ctx *ctx, const madpipe_chain *chain_dev, int32_t P, int64_t M,
                       double beta, const madpipe_disc *disc, madpipe_alloc *out);
 
-/* Multi-GPU building blocks (one process per GPU).
- * madpipe_sweep evaluates this rank's shard of candidates and writes the
- * smallest feasible candidate index it owns (INT32_MAX if none) to *j_local
- * [dev, int32]; the caller min-reduces it across ranks (one NCCL all-reduce,
- * a7) and passes the global minimum to madpipe_resolve [dev, int32], which
- * re-solves that candidate and traces it back; every rank gets the same result.
- * cell_updates_out [host] receives this rank's relaxation count. With
- * disc->early_exit the rank stops at its first feasible candidate. */
+/* The two halves of a multi-GPU solve, for a rank `rank` of `world` given
+ * explicitly (independent of the ctx's own rank/world; no collective): what
+ * madpipe_solve does around its all-reduce, exposed for tests and for callers
+ * with their own transport.  madpipe_sweep evaluates that rank's shard of
+ * candidates and writes the smallest feasible candidate index it owns
+ * (INT32_MAX if none) to *j_local [dev, int32]; the min over ranks, passed to
+ * madpipe_resolve [dev, int32], is re-solved and traced back; every rank gets
+ * the same result.  cell_updates_out [host] receives the shard's relaxation
+ * count.  With disc->early_exit the rank stops at its first feasible candidate. */
 int madpipe_sweep(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int64_t M,
                   double beta, const madpipe_disc *disc, int32_t rank, int32_t world,
                   int32_t *j_local, int64_t *cell_updates_out);
@@ -149,13 +172,45 @@ int madpipe_resolve(madpipe_ctx *ctx, const madpipe_chain *chain, int32_t P, int
                     double beta, const madpipe_disc *disc, const int32_t *j_star,
                     madpipe_alloc *out);
 
-/* Batch of n independent chains (BASELINE config 5) with per-chain P[i],
- * M[i], beta[i] and a shared discretisation; out[i] as for madpipe_solve.
- * All (chain, candidate) pairs run as one sweep. Returns MADPIPE_OK if the call
- * succeeded (each out[i].cand_index is -1 for an infeasible chain). [host]. */
+/* Batch of n independent chains (BASELINE config 5, the paper's evaluation
+ * grid P:235) with per-chain P[i], M[i], beta[i] and a shared discretisation;
+ * out[i] as for madpipe_solve (cand_index -1 for an infeasible chain).  All
+ * (chain, candidate) pairs form one work list.  At world > 1 the list is split
+ * over the ranks by LPT on each pair's cell-update count (madpipe_batch_plan),
+ * the ranks MIN-all-reduce an int32[n] of per-chain smallest feasible indices
+ * (a7), each winner is re-solved by one owner (madpipe_resolve_plan) and the
+ * fixed-size results are all-gathered, so every rank returns all n results.
+ * out[i].cell_updates counts this rank's relaxations of chain i.  Returns
+ * MADPIPE_OK if the call succeeded.  [host]. */
 int madpipe_solve_batch(madpipe_ctx *ctx, int32_t n, const madpipe_chain *chains,
                         const int32_t *P, const int64_t *M, const double *beta,
                         const madpipe_disc *disc, madpipe_alloc *out);
+/* Building blocks of the batch at rank `rank` of `world` (independent of the
+ * ctx's own rank/world; no collective): madpipe_sweep_batch evaluates the jobs
+ * the plan gives this rank and writes j_local[n] [host] (INT32_MAX where this
+ * rank found none) and cell_updates_out[n] [host, may be NULL];
+ * madpipe_resolve_batch re-solves the winners j_star[n] [host] (INT32_MAX =
+ * infeasible) this rank owns and writes only those out[i].  The element-wise
+ * MIN of the ranks' j_local is what madpipe_solve_batch all-reduces. */
+int madpipe_sweep_batch(madpipe_ctx *ctx, int32_t n, const madpipe_chain *chains, const int32_t *P,
+                        const int64_t *M, const double *beta, const madpipe_disc *disc, int32_t rank,
+                        int32_t world, int32_t *j_local, int64_t *cell_updates_out);
+int madpipe_resolve_batch(madpipe_ctx *ctx, int32_t n, const madpipe_chain *chains, const int32_t *P,
+                          const int64_t *M, const double *beta, const madpipe_disc *disc,
+                          const int32_t *j_star, int32_t rank, int32_t world, madpipe_alloc *out);
+/* Host-only (no GPU): the batch work plan over `world` ranks.  owner[n*n_periods]
+ * (may be NULL): owner[i*n_periods + j] = rank evaluating candidate j of chain i;
+ * load[world] (may be NULL): each rank's summed cost; cost[n*n_periods] (may be
+ * NULL): the cost of each pair = its cell-updates + (L+1) n_delay P.
+ * LPT: pairs by decreasing cost (ties: lower index), each to the least-loaded rank
+ * (ties: lower rank); deterministic, so every rank computes the same plan.
+ * madpipe_resolve_plan: owner[n] of each winner's re-solve (LPT on the winners'
+ * costs; -1 where j_star[i] = INT32_MAX). [host] chains (uF, uB, a read). */
+int madpipe_batch_plan(int32_t n, const madpipe_chain *chains, const int32_t *P, const double *beta,
+                       const madpipe_disc *disc, int32_t world, int32_t *owner, int64_t *load,
+                       int64_t *cost);
+int madpipe_resolve_plan(int32_t n, const madpipe_chain *chains, const int32_t *P, const double *beta,
+                         const madpipe_disc *disc, const int32_t *j_star, int32_t world, int32_t *owner);
 
 /* ---- parity / debug exports (small configs) ------------------------------- */
 /* Every candidate's period tau_out[n_periods] and root value root_out[n_periods]
@@ -199,7 +254,7 @@ int madpipe_last_counts(const madpipe_ctx *ctx, int64_t *cell_updates, int64_t *
 int madpipe_last_step_bytes(const madpipe_ctx *ctx, int64_t *load_bytes, int64_t *store_bytes,
                             int64_t *segments);
 /* Step kernel that ran the largest batch of the last sweep:
- * 0 = plain-load step_kernel, 1 = per-tile TMA step_tma_kernel, 2 = persistent
+ * 0 = plain-load step_kernel, 2 = persistent
  * single-layer step_persist_kernel, 3 = persistent two-layer pair_step_kernel.
  * Chosen per batch from the row-segment size unless MADPIPE_KERNEL forces one.
  * Host only. */

@@ -15,8 +15,56 @@ import numpy as np
 from . import _native as N
 from ._native import VRANGE_PAPER, VRANGE_SAFE, MadpipeError  # noqa: F401
 
-__all__ = ["Context", "validate", "shard", "cell_updates", "schedule", "VRANGE_PAPER", "VRANGE_SAFE",
-           "MadpipeError"]
+__all__ = ["Context", "validate", "shard", "cell_updates", "schedule", "get_unique_id", "batch_plan",
+           "resolve_plan", "VRANGE_PAPER", "VRANGE_SAFE", "MadpipeError"]
+
+
+def get_unique_id() -> bytes:
+    """madpipe_get_unique_id: the 128-byte NCCL id one rank creates for the others."""
+    b = ctypes.create_string_buffer(128)
+    N.check(N.lib().madpipe_get_unique_id(b))
+    return b.raw
+
+
+class _Batch:
+    """Keeps the ctypes arrays of a batch of host chains alive for one call."""
+
+    def __init__(self, chains, Ps, Ms, betas):
+        self.hcs = [N.HostChain(c) for c in chains]
+        self.n = len(self.hcs)
+        self.arr = (N.Chain * self.n)(*[h.c for h in self.hcs])
+        self.P = np.ascontiguousarray(Ps, np.int32)
+        self.M = np.ascontiguousarray(Ms if Ms is not None else np.ones(self.n), np.int64)
+        self.B = np.ascontiguousarray(betas, np.float64)
+
+    def args(self):
+        return (self.n, self.arr, self.P.ctypes.data_as(N._i32p), self.M.ctypes.data_as(N._i64p),
+                self.B.ctypes.data_as(N._dp))
+
+
+def batch_plan(chains, Ps, betas, n_mem, n_delay, n_periods, world):
+    """madpipe_batch_plan (host only): (owner[n][n_periods], load[world], cost[n][n_periods])."""
+    b = _Batch(chains, Ps, None, betas)
+    d = N.make_disc(n_mem, n_delay, n_periods)
+    owner = np.empty((b.n, n_periods), np.int32)
+    load = np.empty(world, np.int64)
+    cost = np.empty((b.n, n_periods), np.int64)
+    N.check(N.lib().madpipe_batch_plan(b.n, b.arr, b.P.ctypes.data_as(N._i32p), b.B.ctypes.data_as(N._dp),
+                                       ctypes.byref(d), int(world), owner.ctypes.data_as(N._i32p),
+                                       load.ctypes.data_as(N._i64p), cost.ctypes.data_as(N._i64p)))
+    return owner, load, cost
+
+
+def resolve_plan(chains, Ps, betas, n_mem, n_delay, n_periods, j_star, world):
+    """madpipe_resolve_plan (host only): the rank re-solving each chain's winner (-1: none)."""
+    b = _Batch(chains, Ps, None, betas)
+    d = N.make_disc(n_mem, n_delay, n_periods)
+    js = np.ascontiguousarray(j_star, np.int32)
+    owner = np.empty(b.n, np.int32)
+    N.check(N.lib().madpipe_resolve_plan(b.n, b.arr, b.P.ctypes.data_as(N._i32p), b.B.ctypes.data_as(N._dp),
+                                         ctypes.byref(d), js.ctypes.data_as(N._i32p), int(world),
+                                         owner.ctypes.data_as(N._i32p)))
+    return owner
 
 
 def validate(chain, P, M, beta, n_mem, n_delay, n_periods, v_range=VRANGE_PAPER) -> int:
@@ -76,17 +124,27 @@ def _any_chain(chain):
 
 
 class Context:
-    """A libmadpipe context bound to one CUDA device (madpipe_ctx_create)."""
+    """A libmadpipe context bound to one CUDA device (madpipe_ctx_create): rank ``rank`` of
+    ``world``; with ``nccl_id`` (128 bytes, see distributed.context) the ctx owns the NCCL
+    communicator its solves all-reduce over."""
 
-    def __init__(self, device: int = 0, stream=None, mem_budget: int = 0):
+    def __init__(self, device: int = 0, stream=None, mem_budget: int = 0, rank: int = 0, world: int = 1,
+                 nccl_id: bytes | None = None):
         self._lib = N.lib()
         h = ctypes.c_void_p()
-        rc = self._lib.madpipe_ctx_create(ctypes.byref(h), int(device),
-                                          ctypes.c_void_p(stream) if stream else None, int(mem_budget))
+        rc = self._lib.madpipe_ctx_create(ctypes.byref(h), int(device), int(rank), int(world),
+                                          nccl_id, ctypes.c_void_p(stream) if stream else None,
+                                          int(mem_budget))
         if rc != N.OK:
             raise MadpipeError(rc, N.last_error(None))
         self.h = h
         self.device = device
+        self.rank, self.world = int(rank), int(world)
+
+    def info(self):
+        r = ctypes.c_int32(); w = ctypes.c_int32(); v = ctypes.c_int32()
+        N.check(self._lib.madpipe_ctx_info(self.h, ctypes.byref(r), ctypes.byref(w), ctypes.byref(v)))
+        return dict(rank=r.value, world=w.value, nccl_version=v.value)
 
     def close(self):
         if getattr(self, "h", None):
@@ -154,22 +212,49 @@ class Context:
 
     def solve_batch(self, chains, Ps, Ms, betas, n_mem, n_delay, n_periods, v_range=VRANGE_PAPER,
                     early_exit=False):
-        hcs = [N.HostChain(c) for c in chains]
-        n = len(hcs)
-        arr = (N.Chain * n)(*[h.c for h in hcs])
-        P = np.ascontiguousarray(Ps, np.int32)
-        M = np.ascontiguousarray(Ms, np.int64)
-        B = np.ascontiguousarray(betas, np.float64)
-        bufs = [N.AllocBuf(h.L) for h in hcs]
-        outs = (N.Alloc * n)(*[b.s for b in bufs])
+        b = _Batch(chains, Ps, Ms, betas)
+        bufs = [N.AllocBuf(h.L) for h in b.hcs]
+        outs = (N.Alloc * b.n)(*[x.s for x in bufs])
         d = N.make_disc(n_mem, n_delay, n_periods, v_range, early_exit)
-        N.check(self._lib.madpipe_solve_batch(self.h, n, arr, P.ctypes.data_as(N._i32p),
-                                              M.ctypes.data_as(N._i64p), B.ctypes.data_as(N._dp),
-                                              ctypes.byref(d), outs), self.h)
+        N.check(self._lib.madpipe_solve_batch(self.h, *b.args(), ctypes.byref(d), outs), self.h)
+        return self._batch_results(bufs, outs)
+
+    @staticmethod
+    def _batch_results(bufs, outs):
         res = []
-        for b, o in zip(bufs, outs):
-            b.s = o
-            res.append(b.result(N.OK if o.cand_index >= 0 else N.INFEASIBLE))
+        for x, o in zip(bufs, outs):
+            x.s = o
+            res.append(x.result(N.OK if o.cand_index >= 0 else N.INFEASIBLE))
+        return res
+
+    def sweep_batch(self, chains, Ps, Ms, betas, n_mem, n_delay, n_periods, rank, world, v_range=VRANGE_PAPER,
+                    early_exit=False):
+        """madpipe_sweep_batch: (j_local[n], cell_updates[n]) of rank ``rank`` of ``world``."""
+        b = _Batch(chains, Ps, Ms, betas)
+        d = N.make_disc(n_mem, n_delay, n_periods, v_range, early_exit)
+        jl = np.empty(b.n, np.int32)
+        cu = np.empty(b.n, np.int64)
+        N.check(self._lib.madpipe_sweep_batch(self.h, *b.args(), ctypes.byref(d), int(rank), int(world),
+                                              jl.ctypes.data_as(N._i32p), cu.ctypes.data_as(N._i64p)), self.h)
+        return jl, cu
+
+    def resolve_batch(self, chains, Ps, Ms, betas, n_mem, n_delay, n_periods, j_star, rank, world,
+                      v_range=VRANGE_PAPER):
+        """madpipe_resolve_batch: results of the winners rank ``rank`` owns ({chain: result})."""
+        b = _Batch(chains, Ps, Ms, betas)
+        d = N.make_disc(n_mem, n_delay, n_periods, v_range)
+        js = np.ascontiguousarray(j_star, np.int32)
+        bufs = [N.AllocBuf(h.L) for h in b.hcs]
+        for x in bufs:
+            x.s.cand_index = -2                      # marks "not written by this rank"
+        outs = (N.Alloc * b.n)(*[x.s for x in bufs])
+        N.check(self._lib.madpipe_resolve_batch(self.h, *b.args(), ctypes.byref(d), js.ctypes.data_as(N._i32p),
+                                                int(rank), int(world), outs), self.h)
+        res = {}
+        for i, (x, o) in enumerate(zip(bufs, outs)):
+            if o.cand_index != -2:
+                x.s = o
+                res[i] = x.result(N.OK if o.cand_index >= 0 else N.INFEASIBLE)
         return res
 
     # ------------------------------------------------------------------ parity exports
@@ -242,7 +327,7 @@ class Context:
         """Step kernel of the largest batch of the last sweep (madpipe_last_kernel)."""
         k = ctypes.c_int32()
         N.check(self._lib.madpipe_last_kernel(self.h, ctypes.byref(k)))
-        return {0: "step_kernel", 1: "step_tma_kernel", 2: "step_persist_kernel",
+        return {0: "step_kernel", 2: "step_persist_kernel",
                 3: "pair_step_kernel"}.get(k.value, None)
 
     def last_timing(self):

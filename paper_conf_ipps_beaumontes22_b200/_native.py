@@ -12,7 +12,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 # MADPIPE_LIB: an alternative in-tree build (A/B experiments, build.py MADPIPE_DEFS)
 LIB_PATH = os.environ.get("MADPIPE_LIB") or os.path.join(_HERE, "libmadpipe.so")
 
-OK, INFEASIBLE, EINVAL, ENOMEM, ECUDA, ESTATE = 0, 1, -1, -2, -3, -5
+OK, INFEASIBLE, EINVAL, ENOMEM, ECUDA, ENCCL, ESTATE = 0, 1, -1, -2, -3, -4, -5
 VRANGE_PAPER, VRANGE_SAFE = 0, 1
 
 _i32p = ctypes.POINTER(ctypes.c_int32)
@@ -62,7 +62,10 @@ def lib():
     dcp = ctypes.POINTER(Disc)
     ap = ctypes.POINTER(Alloc)
     sig = {
-        "madpipe_ctx_create": (ctypes.c_int, [ctypes.POINTER(vp), ctypes.c_int, vp, ctypes.c_int64]),
+        "madpipe_get_unique_id": (ctypes.c_int, [ctypes.c_char_p]),
+        "madpipe_ctx_create": (ctypes.c_int, [ctypes.POINTER(vp), ctypes.c_int, ctypes.c_int32, ctypes.c_int32,
+                                              ctypes.c_char_p, vp, ctypes.c_int64]),
+        "madpipe_ctx_info": (ctypes.c_int, [vp, _i32p, _i32p, _i32p]),
         "madpipe_ctx_destroy": (None, [vp]),
         "madpipe_last_error": (ctypes.c_char_p, [vp]),
         "madpipe_validate": (ctypes.c_int, [cp, ctypes.c_int32, ctypes.c_int64, ctypes.c_double, dcp]),
@@ -75,6 +78,14 @@ def lib():
         "madpipe_resolve": (ctypes.c_int, [vp, cp, ctypes.c_int32, ctypes.c_int64, ctypes.c_double, dcp,
                                            vp, ap]),
         "madpipe_solve_batch": (ctypes.c_int, [vp, ctypes.c_int32, cp, _i32p, _i64p, _dp, dcp, ap]),
+        "madpipe_sweep_batch": (ctypes.c_int, [vp, ctypes.c_int32, cp, _i32p, _i64p, _dp, dcp, ctypes.c_int32,
+                                               ctypes.c_int32, _i32p, _i64p]),
+        "madpipe_resolve_batch": (ctypes.c_int, [vp, ctypes.c_int32, cp, _i32p, _i64p, _dp, dcp, _i32p,
+                                                 ctypes.c_int32, ctypes.c_int32, ap]),
+        "madpipe_batch_plan": (ctypes.c_int, [ctypes.c_int32, cp, _i32p, _dp, dcp, ctypes.c_int32, _i32p, _i64p,
+                                              _i64p]),
+        "madpipe_resolve_plan": (ctypes.c_int, [ctypes.c_int32, cp, _i32p, _dp, dcp, _i32p, ctypes.c_int32,
+                                                _i32p]),
         "madpipe_candidates": (ctypes.c_int, [vp, cp, ctypes.c_int32, ctypes.c_int64, ctypes.c_double,
                                               dcp, _dp, _dp]),
         "madpipe_dp_table": (ctypes.c_int, [vp, cp, ctypes.c_int32, ctypes.c_int64, ctypes.c_double,
@@ -102,9 +113,11 @@ def lib():
     return _lib
 
 
-EXPORTED = ["madpipe_ctx_create", "madpipe_ctx_destroy", "madpipe_last_error", "madpipe_validate",
+EXPORTED = ["madpipe_get_unique_id", "madpipe_ctx_create", "madpipe_ctx_destroy", "madpipe_ctx_info",
+            "madpipe_last_error", "madpipe_validate",
             "madpipe_shard", "madpipe_cell_updates", "madpipe_solve", "madpipe_solve_dev",
-            "madpipe_sweep", "madpipe_resolve", "madpipe_solve_batch", "madpipe_candidates",
+            "madpipe_sweep", "madpipe_resolve", "madpipe_solve_batch", "madpipe_sweep_batch",
+            "madpipe_resolve_batch", "madpipe_batch_plan", "madpipe_resolve_plan", "madpipe_candidates",
             "madpipe_dp_table", "madpipe_last_timing", "madpipe_set_timing", "madpipe_last_io",
             "madpipe_last_counts", "madpipe_last_step_bytes", "madpipe_last_kernel", "madpipe_schedule", "madpipe_solve_paper", "madpipe_literal_table"]
 

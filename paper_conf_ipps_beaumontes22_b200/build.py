@@ -14,7 +14,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.environ.get("MADPIPE_LIB") or os.path.join(HERE, "libmadpipe.so")
-SOURCES = ["mp_kernels.cu", "mp_step_tma.cu", "mp_step_persist.cu", "mp_step_pair.cu", "mp_api.cu", "mp_schedule.cu", "mp_literal.cu"]
+SOURCES = ["mp_kernels.cu", "mp_step_persist.cu", "mp_step_pair.cu", "mp_api.cu", "mp_schedule.cu", "mp_literal.cu", "mp_comm.cu"]
 HEADERS = ["mp_internal.cuh", "mp_device.cuh", os.path.join("..", "..", "include", "madpipe.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -22,8 +22,17 @@ FLAGS = ["-O3", "-std=c++17", "-lineinfo", "--fmad=false", "-Xcompiler", "-fPIC,
          "-Xptxas", "-v"] + os.environ.get("MADPIPE_DEFS", "").split()   # A/B experiment macros
 
 
+def _defs_stamp() -> str:
+    return " ".join(FLAGS)
+
+
 def _stale() -> bool:
+    """Rebuild when a source is newer than the library or when the library was built
+    with other flags (MADPIPE_DEFS variants: the flags are stamped next to it)."""
     if not os.path.exists(LIB):
+        return True
+    stamp = LIB + ".flags"
+    if not os.path.exists(stamp) or open(stamp).read() != _defs_stamp():
         return True
     t = os.path.getmtime(LIB)
     deps = [os.path.join(CSRC, f) for f in SOURCES + HEADERS] + [os.path.abspath(__file__)]
@@ -45,12 +54,14 @@ def build(force: bool = False, verbose: bool = False) -> str:
             sys.stderr.write(r.stderr)
         objs.append(obj)
     tmp = LIB + ".tmp.%d" % os.getpid()
-    cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart_static", "-lrt", "-ldl", "-lpthread"]
+    cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart_static", "-lrt", "-ldl", "-lpthread"]   # NCCL: dlopen (mp_comm.cu)
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
         raise RuntimeError("nvcc link failed")
     os.replace(tmp, LIB)
+    with open(LIB + ".flags", "w") as f:
+        f.write(_defs_stamp())
     for o in objs:
         os.remove(o)
     return LIB

@@ -5,6 +5,7 @@
 // only validates arguments, moves the O(L) profile to the device, lays out the
 // DP tables in HBM and issues the launches (DESIGN.md sections 6-7).
 #include <algorithm>
+#include <numeric>
 #include <chrono>
 #include <climits>
 #include <cmath>
@@ -55,7 +56,7 @@ struct madpipe_ctx {
     int64_t last_cell_updates = 0, last_effective = 0, last_useful = 0, last_segs = 0;
     int64_t last_load_bytes = 0, last_store_bytes = 0;   // step kernel: source segments in, rows out
     int per_launch_timing = 0;
-    int kernel = -1;          // MADPIPE_KERNEL: v1 = plain loads, tma = per-tile TMA, persist, pair;
+    int kernel = -1;          // MADPIPE_KERNEL: v1 = plain loads, persist, pair (1 = retired per-tile TMA);
                               // -1 (default): pair for P > 33 (n_mem <= 8), else persist
                               // when a row segment is >= 1 KB, else v1
     int prof = 0;             // MADPIPE_PROF=1: cycle counters of the persistent step kernel to stderr
@@ -67,6 +68,11 @@ struct madpipe_ctx {
     int last_kernel = -1;     // step kernel of the largest batch of the last timed sweep
     int last_kernel_jobs = 0;
     std::vector<cudaEvent_t> ev_pool;
+    // multi-GPU: this process's rank of `world`, and the NCCL communicator
+    // over which a7 (the min-reduction) and the batch's result all-gather run
+    int32_t rank = 0, world = 1;
+    void *comm = nullptr;
+    DevBuf gather;
 };
 
 static thread_local std::string g_err;
@@ -205,10 +211,19 @@ extern "C" const char *madpipe_last_error(const madpipe_ctx *ctx) {
 // ---------------------------------------------------------------------------
 // context
 // ---------------------------------------------------------------------------
-extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stream,
-                                  int64_t mem_budget) {
+extern "C" int madpipe_get_unique_id(uint8_t id[128]) {
+    if (!id) return fail(nullptr, MADPIPE_EINVAL, "null id");
+    std::string why;
+    if (comm_unique_id(id, &why)) return fail(nullptr, MADPIPE_ENCCL, "%s", why.c_str());
+    return MADPIPE_OK;
+}
+
+extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, int32_t rank, int32_t world,
+                                  const uint8_t *nccl_id, void *cuda_stream, int64_t mem_budget) {
     if (!out) return fail(nullptr, MADPIPE_EINVAL, "null out");
     *out = nullptr;
+    if (world < 1 || rank < 0 || rank >= world) return fail(nullptr, MADPIPE_EINVAL, "bad rank %d / world %d", rank, world);
+    if (world > 1 && !nccl_id) return fail(nullptr, MADPIPE_EINVAL, "world > 1 needs an NCCL id");
     int n = 0;
     cudaError_t e = cudaGetDeviceCount(&n);
     if (e != cudaSuccess || n == 0)
@@ -218,10 +233,20 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stre
     if (e != cudaSuccess) return fail(nullptr, MADPIPE_ECUDA, "cudaSetDevice: %s", cudaGetErrorString(e));
     madpipe_ctx *c = new madpipe_ctx();
     c->device = device;
+    c->rank = rank;
+    c->world = world;
+    if (nccl_id) {
+        std::string why;
+        if (comm_init(&c->comm, world, rank, nccl_id, &why)) {
+            delete c;
+            return fail(nullptr, MADPIPE_ENCCL, "%s", why.c_str());
+        }
+    }
     if (cuda_stream) {
         c->stream = (cudaStream_t)cuda_stream;
     } else {
         if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess) {
+            comm_destroy(c->comm);
             delete c;
             return fail(nullptr, MADPIPE_ECUDA, "cudaStreamCreate failed");
         }
@@ -232,7 +257,6 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, void *cuda_stre
     c->mem_budget = mem_budget > 0 ? mem_budget : (int64_t)(0.6 * (double)fr);
     const char *kern = getenv("MADPIPE_KERNEL");
     if (kern && strcmp(kern, "v1") == 0) c->kernel = 0;
-    if (kern && strcmp(kern, "tma") == 0) c->kernel = 1;
     if (kern && strcmp(kern, "persist") == 0) c->kernel = 2;
     if (kern && strcmp(kern, "pair") == 0) c->kernel = 3;
     cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device);
@@ -271,7 +295,17 @@ extern "C" void madpipe_ctx_destroy(madpipe_ctx *c) {
     if (c->ev_a) cudaEventDestroy(c->ev_a);
     if (c->ev_b) cudaEventDestroy(c->ev_b);
     if (c->own_stream) cudaStreamDestroy(c->stream);
+    c->gather.release();
+    comm_destroy(c->comm);
     delete c;
+}
+
+extern "C" int madpipe_ctx_info(const madpipe_ctx *c, int32_t *rank, int32_t *world, int32_t *nccl_version) {
+    if (!c) return MADPIPE_EINVAL;
+    if (rank) *rank = c->rank;
+    if (world) *world = c->world;
+    if (nccl_version) *nccl_version = c->comm ? comm_version() : 0;
+    return MADPIPE_OK;
 }
 
 extern "C" int madpipe_last_timing(const madpipe_ctx *c, double *sweep_ms, double *step_ms,
@@ -434,6 +468,8 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
     // early exit: small first batches that double (time-to-placement); otherwise as
     // many jobs as the table budget holds
     size_t cap_jobs = early_exit ? (size_t)8 * (size_t)n_chains : SIZE_MAX;
+    int all_maxL = 1;
+    for (const auto &c : cs) all_maxL = std::max(all_maxL, (int)c.c.L);
     while (next < js.size()) {
         // ---- form a batch
         hjobs.clear(); htiles.clear(); ids.clear();
@@ -441,7 +477,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         // one row segment per stage, which pays off from ~1 KB segments; below, plain loads win
         int kern = ctx->kernel;
         while (next < js.size() && early_exit && jl_host[js[next].chain] < js[next].j) next++;
-        if (kern == 3 && next < js.size() && !pair_supported(cs[js[next].chain].P, nmp, disc->n_delay)) kern = -1;
+        if (kern == 3 && next < js.size() && !pair_supported(cs[js[next].chain].P, nmp, disc->n_delay, all_maxL)) kern = -1;
         if (kern < 0 && next < js.size()) {
             int vb_, np_, npt_, nt_;
             persist_geom(cs[js[next].chain].P, disc->n_delay, nmp, &vb_, &np_, &npt_, &nt_);
@@ -450,12 +486,11 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             // profiles/r01_pair_dispatch.md): P > 33 (the single-layer kernel needs two
             // warps per delay row there), n_mem <= 8
             const int P = cs[js[next].chain].P;
-            if (P > 33 && pair_supported(P, nmp, disc->n_delay)) kern = 3;
+            if (P > 33 && pair_supported(P, nmp, disc->n_delay, all_maxL)) kern = 3;
         }
         size_t used = 0;
         int maxL = 0;
         size_t max_slab = 0;
-        int smem_tma = 0;
         for (; next < js.size(); next++) {
             const JobSpec &s = js[next];
             if (early_exit && jl_host[s.chain] < s.j) continue;
@@ -482,9 +517,6 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 J.vb = 0;
             } else if (kern == 2) {
                 persist_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
-            } else if (kern == 1) {
-                tma_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
-                smem_tma = std::max(smem_tma, tma_smem_bytes(J.vb, J.np, nmp));
             } else {
                 tile_geom(c.P, disc->n_delay, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
             }
@@ -695,8 +727,6 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 launch_step_persist(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, p_np, p_vb, nsg,
                                     persist_grid, (unsigned long long *)(ctx->prof ? ctx->profbuf.p : nullptr),
                                     ctx->n_prod, ctx->tile_block, buf_off, ctx->stream);
-            else if (kern == 1)
-                launch_step_tma(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, smem_tma, ctx->stream);
             else
                 launch_step(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, ctx->stream);
             if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1) + 1], ctx->stream);
@@ -899,6 +929,16 @@ std::vector<JobSpec> shard_jobs(int chain, int n_c, int rank, int world) {
     return js;
 }
 
+// a7: min-reduce n int32 candidate indices (device) over the ctx's communicator, on
+// the ctx's stream.  Without a communicator (world 1) this is the identity.
+int allreduce_min(madpipe_ctx *ctx, int32_t *dev, size_t n) {
+    if (!ctx->comm) return MADPIPE_OK;
+    std::string why;
+    if (comm_allreduce_min_i32(ctx->comm, dev, n, ctx->stream, &why))
+        return fail(ctx, MADPIPE_ENCCL, "%s", why.c_str());
+    return MADPIPE_OK;
+}
+
 int solve_common(madpipe_ctx *ctx, const madpipe_chain *chain, bool on_device, int32_t P, int64_t M,
                  double beta, const madpipe_disc *disc, madpipe_alloc *out) {
     int rc = begin(ctx);
@@ -913,18 +953,27 @@ int solve_common(madpipe_ctx *ctx, const madpipe_chain *chain, bool on_device, i
     CUDA_TRY(ctx, ctx->jl.ensure(sizeof(int32_t)));
     int64_t cu = 0;
     int32_t jstar = INT32_MAX;
-    // evaluate a list of candidates (ascending), smallest feasible index -> jstar
+    const int R = ctx->rank, W = ctx->world;
+    // One round: this rank evaluates its share of `js` (ascending; with `early`, it stops
+    // at its first feasible candidate -- exact, a smaller feasible index always wins),
+    // then the ranks min-reduce their smallest feasible index (a7, one all-reduce).
     auto sweep = [&](const std::vector<JobSpec> &js, bool early, double *ms_acc, double *kern_acc,
                      int64_t *eff_acc, int64_t *useful_acc) -> int {
         int r = fill_int_max(ctx, (int32_t *)ctx->jl.p, 1);
         if (r) return r;
+        std::vector<JobSpec> mine;
+        for (size_t i = (size_t)R; i < js.size(); i += (size_t)W) mine.push_back(js[i]);
         std::vector<uint64_t> counts;
-        r = run_jobs(ctx, cs, cd, disc, js, (int32_t *)ctx->jl.p, nullptr, nullptr, &counts, early, nullptr,
-                     true);
+        if (!mine.empty()) {
+            r = run_jobs(ctx, cs, cd, disc, mine, (int32_t *)ctx->jl.p, nullptr, nullptr, &counts, early, nullptr,
+                         true);
+            if (r) return r;
+            for (auto x : counts) cu += (int64_t)x;
+            *ms_acc += ctx->sweep_ms; *kern_acc += ctx->step_ms;
+            *eff_acc += ctx->last_effective; *useful_acc += ctx->last_useful;
+        }
+        r = allreduce_min(ctx, (int32_t *)ctx->jl.p, 1);
         if (r) return r;
-        for (auto x : counts) cu += (int64_t)x;
-        *ms_acc += ctx->sweep_ms; *kern_acc += ctx->step_ms;
-        *eff_acc += ctx->last_effective; *useful_acc += ctx->last_useful;
         int32_t j = INT32_MAX;
         CUDA_TRY(ctx, d2h(ctx, &j, ctx->jl.p, sizeof(int32_t)));
         CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
@@ -936,8 +985,9 @@ int solve_common(madpipe_ctx *ctx, const madpipe_chain *chain, bool on_device, i
     const int n_c = disc->n_periods;
     if (disc->early_exit == 2 && n_c > 4) {
         // NEXT row f3, coarse-to-fine: every s-th candidate in ascending order until one is
-        // feasible (J1), then the candidates of the gap (J1-s, J1).  Exact when feasibility is
-        // monotone in the period; early_exit = 1 is exact without that assumption.
+        // feasible (J1), then the candidates of the gap (J1-s, J1); each round is split over
+        // the ranks and ends in one all-reduce.  Exact when feasibility is monotone in the
+        // period; early_exit = 1 is exact without that assumption.
         const int step = std::max(2, (int)std::lround(std::sqrt((double)n_c)));
         std::vector<JobSpec> coarse;
         for (int j = 0; j < n_c; j += step) coarse.push_back({0, j});
@@ -964,10 +1014,168 @@ int solve_common(madpipe_ctx *ctx, const madpipe_chain *chain, bool on_device, i
         fill_infeasible(out, cu);
         return MADPIPE_INFEASIBLE;
     }
+    // a8: every rank re-solves the winner and traces it back (deterministic: no broadcast)
     std::vector<int32_t> js{jstar};
     rc = resolve_impl(ctx, cs, cd, disc, js, out);
     out->cell_updates = cu;
     return rc;
+}
+
+// ---------------------------------------------------------------------------
+// batch work plan: LPT over the (chain, candidate) work list
+// ---------------------------------------------------------------------------
+// Host estimate of the cost of job (chain, j): its cell-updates at tau_j,
+// sum_l (l - kmin(l) + 1) (P-1) n_v n_m, with the same prefix sums and grid formula as
+// prep_kernel / jobs_init_kernel.  Only used to balance ranks; identical on every rank.
+void batch_costs(const std::vector<ChainSpec> &cs, const madpipe_disc *disc, std::vector<int64_t> &cost) {
+    const int n_c = disc->n_periods;
+    cost.assign(cs.size() * (size_t)n_c, 0);
+    std::vector<double> Up;
+    for (size_t c = 0; c < cs.size(); c++) {
+        const madpipe_chain &ch = cs[c].c;
+        const int L = ch.L, P = cs[c].P;
+        Up.assign(L + 1, 0.0);
+        for (int i = 1; i <= L; i++) Up[i] = Up[i - 1] + (ch.uF[i - 1] + ch.uB[i - 1]);
+        double SC = 0.0;
+        for (int i = 1; i <= L - 1; i++) SC = SC + (2.0 * (double)ch.a[i]) / cs[c].beta;
+        const double lb = Up[L] / (double)P, ub = Up[L] + SC;
+        const int64_t per = (int64_t)std::max(0, P - 1) * disc->n_delay * disc->n_mem;
+        for (int j = 0; j < n_c; j++) {
+            const double tau = n_c == 1 ? ub : lb + (double)j * ((ub - lb) / (double)(n_c - 1));
+            int64_t t = 0;
+            int k = 1;
+            for (int l = 1; l <= L; l++) {
+                while (k <= l && Up[l] - Up[k - 1] > tau) k++;
+                if (k <= l) t += (int64_t)(l - k + 1);
+            }
+            // + one (L+1) x n_v x P row sweep of fixed work per job (init, trans, roots)
+            cost[c * (size_t)n_c + j] = t * per + (int64_t)(L + 1) * disc->n_delay * P;
+        }
+    }
+}
+
+// Longest-processing-time-first: items by decreasing cost (ties: lower index first),
+// each to the rank with the smallest load so far (ties: lower rank).  Deterministic.
+void lpt(const std::vector<int64_t> &cost, const std::vector<int32_t> &items, int world, std::vector<int32_t> &owner,
+         std::vector<int64_t> *load_out) {
+    std::vector<int32_t> order(items);
+    std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) { return cost[a] > cost[b]; });
+    std::vector<int64_t> load(world, 0);
+    for (int32_t it : order) {
+        int best = 0;
+        for (int r = 1; r < world; r++) if (load[r] < load[best]) best = r;
+        owner[it] = best;
+        load[best] += cost[it];
+    }
+    if (load_out) *load_out = load;
+}
+
+// owner[c * n_c + j] = rank that evaluates candidate j of chain c
+void batch_plan(const std::vector<ChainSpec> &cs, const madpipe_disc *disc, int world, std::vector<int32_t> &owner,
+                std::vector<int64_t> *load, std::vector<int64_t> *cost_out) {
+    std::vector<int64_t> cost;
+    batch_costs(cs, disc, cost);
+    owner.assign(cost.size(), 0);
+    std::vector<int32_t> items(cost.size());
+    for (size_t i = 0; i < items.size(); i++) items[i] = (int32_t)i;
+    if (world > 1) lpt(cost, items, world, owner, load);
+    else if (load) load->assign(1, std::accumulate(cost.begin(), cost.end(), (int64_t)0));
+    if (cost_out) *cost_out = std::move(cost);
+}
+
+// rowner[c] = rank that re-solves chain c's winner j*[c] (LPT on the winners' costs); -1 if none
+void resolve_plan(const std::vector<int64_t> &cost, int n_c, const std::vector<int32_t> &jstar, int world,
+                  std::vector<int32_t> &rowner) {
+    const int n = (int)jstar.size();
+    rowner.assign(n, -1);
+    std::vector<int64_t> wc(n, 0);
+    std::vector<int32_t> items;
+    for (int c = 0; c < n; c++)
+        if (jstar[c] != INT32_MAX && jstar[c] >= 0) { items.push_back(c); wc[c] = cost[(size_t)c * n_c + jstar[c]]; }
+    std::vector<int32_t> own(n, -1);
+    if (world > 1) lpt(wc, items, world, own, nullptr);
+    else for (int c : items) own[c] = 0;
+    for (int c : items) rowner[c] = own[c];
+}
+
+int prepare_batch(madpipe_ctx *ctx, int32_t n, const madpipe_chain *chains, const int32_t *P, const int64_t *M,
+                  const double *beta, const madpipe_disc *disc, std::vector<ChainSpec> &cs) {
+    if (n < 1 || !chains || !P || !M || !beta || !disc)
+        return fail(ctx, MADPIPE_EINVAL, "bad batch arguments");
+    for (int i = 0; i < n; i++) {
+        int rc = check_one(ctx, &chains[i], P[i], M[i], beta[i], disc, true);
+        if (rc) return fail(ctx, rc, "chain %d: %s", i, ctx->err.c_str());
+        cs.push_back({chains[i], false, P[i], M[i], beta[i]});
+    }
+    return MADPIPE_OK;
+}
+
+// This rank's share of the batch sweep: jl_dev[c] <- smallest feasible candidate of chain
+// c among the jobs this rank owns (INT32_MAX if none); cu[c] <- this rank's cell-updates.
+int batch_sweep(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vector<ChainDev> &cd,
+                const madpipe_disc *disc, int rank, int world, const std::vector<int32_t> &owner,
+                std::vector<int64_t> &cu) {
+    const int n = (int)cs.size(), n_c = disc->n_periods;
+    CUDA_TRY(ctx, ctx->jl.ensure(sizeof(int32_t) * n));
+    { int _r = fill_int_max(ctx, (int32_t *)ctx->jl.p, n); if (_r) return _r; }
+    // candidate-major order keeps small (cheap) periods of every chain first, so early
+    // exit prunes the expensive large periods
+    std::vector<JobSpec> js;
+    for (int j = 0; j < n_c; j++)
+        for (int c = 0; c < n; c++)
+            if (world == 1 || owner[(size_t)c * n_c + j] == rank) js.push_back({c, j});
+    // group by P (a step launch runs one tile geometry); within a group candidate-major
+    std::stable_sort(js.begin(), js.end(),
+                     [&](const JobSpec &a, const JobSpec &b) { return cs[a.chain].P < cs[b.chain].P; });
+    cu.assign(n, 0);
+    if (js.empty()) return MADPIPE_OK;
+    std::vector<uint64_t> counts;
+    int rc = run_jobs(ctx, cs, cd, disc, js, (int32_t *)ctx->jl.p, nullptr, nullptr, &counts,
+                      disc->early_exit != 0, nullptr, true);
+    if (rc) return rc;
+    for (size_t i = 0; i < js.size(); i++) cu[js[i].chain] += (int64_t)counts[i];
+    return MADPIPE_OK;
+}
+
+// Re-solve and trace back the winners this rank owns (rowner[c] == rank); out[c] of the
+// other chains is left untouched.
+int batch_resolve(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vector<ChainDev> &cd,
+                  const madpipe_disc *disc, const std::vector<int32_t> &jstar, const std::vector<int32_t> &rowner,
+                  int rank, madpipe_alloc *out) {
+    std::vector<int32_t> mine(jstar.size(), INT32_MAX);
+    bool any = false;
+    for (size_t c = 0; c < jstar.size(); c++)
+        if (rowner[c] == rank) { mine[c] = jstar[c]; any = true; }
+    if (!any) return MADPIPE_OK;
+    return resolve_impl(ctx, cs, cd, disc, mine, out);
+}
+
+// Fixed-size int32 record of one chain's result for the all-gather:
+// [period, load_period, special_load as 2 words each][cand_index][n_stages][first|last|proc x Lmax]
+constexpr int kRecHead = 8;
+void pack_rec(const madpipe_alloc &o, int Lmax, int32_t *r) {
+    memcpy(r, &o.period, 8);
+    memcpy(r + 2, &o.load_period, 8);
+    memcpy(r + 4, &o.special_load, 8);
+    r[6] = o.cand_index;
+    r[7] = o.n_stages;
+    for (int s = 0; s < o.n_stages; s++) {
+        r[kRecHead + s] = o.stage_first[s];
+        r[kRecHead + Lmax + s] = o.stage_last[s];
+        r[kRecHead + 2 * Lmax + s] = o.stage_proc[s];
+    }
+}
+void unpack_rec(const int32_t *r, int Lmax, madpipe_alloc &o) {
+    memcpy(&o.period, r, 8);
+    memcpy(&o.load_period, r + 2, 8);
+    memcpy(&o.special_load, r + 4, 8);
+    o.cand_index = r[6];
+    o.n_stages = r[7];
+    for (int s = 0; s < o.n_stages; s++) {
+        if (o.stage_first) o.stage_first[s] = r[kRecHead + s];
+        if (o.stage_last) o.stage_last[s] = r[kRecHead + Lmax + s];
+        if (o.stage_proc) o.stage_proc[s] = r[kRecHead + 2 * Lmax + s];
+    }
 }
 
 }  // namespace
@@ -1044,40 +1252,163 @@ extern "C" int madpipe_solve_batch(madpipe_ctx *ctx, int32_t n, const madpipe_ch
                                    const madpipe_disc *disc, madpipe_alloc *out) {
     int rc = begin(ctx);
     if (rc) return rc;
-    if (n < 1 || !chains || !P || !M || !beta || !out)
-        return fail(ctx, MADPIPE_EINVAL, "bad batch arguments");
+    if (!out) return fail(ctx, MADPIPE_EINVAL, "null out");
     std::vector<ChainSpec> cs;
-    for (int i = 0; i < n; i++) {
-        rc = check_one(ctx, &chains[i], P[i], M[i], beta[i], disc, true);
-        if (rc) return fail(ctx, rc, "chain %d: %s", i, ctx->err.c_str());
-        cs.push_back({chains[i], false, P[i], M[i], beta[i]});
-    }
+    rc = prepare_batch(ctx, n, chains, P, M, beta, disc, cs);
+    if (rc) return rc;
+    const int R = ctx->rank, W = ctx->world, n_c = disc->n_periods;
+    // the same deterministic plan on every rank (identical inputs, SPMD)
+    std::vector<int32_t> owner;
+    std::vector<int64_t> cost;
+    if (W > 1 || ctx->comm) batch_plan(cs, disc, W, owner, nullptr, &cost);
     std::vector<ChainDev> cd;
     rc = upload_chains(ctx, cs, cd);
     if (rc) return rc;
-    CUDA_TRY(ctx, ctx->jl.ensure(sizeof(int32_t) * n));
-    { int _r = fill_int_max(ctx, (int32_t *)ctx->jl.p, n); if (_r) return _r; }
-    // candidate-major order keeps small (cheap) periods of every chain first,
-    // so early exit prunes the expensive large periods
-    std::vector<JobSpec> js;
-    for (int j = 0; j < disc->n_periods; j++)
-        for (int c = 0; c < n; c++) js.push_back({c, j});
-    // group by P (the persistent step kernel launches one tile geometry at a time);
-    // within a group the order stays candidate-major
-    std::stable_sort(js.begin(), js.end(),
-                     [&](const JobSpec &a, const JobSpec &b) { return cs[a.chain].P < cs[b.chain].P; });
-    std::vector<uint64_t> counts;
-    rc = run_jobs(ctx, cs, cd, disc, js, (int32_t *)ctx->jl.p, nullptr, nullptr, &counts,
-                  disc->early_exit != 0, nullptr, true);
+    std::vector<int64_t> cu;
+    rc = batch_sweep(ctx, cs, cd, disc, R, W, owner, cu);
     if (rc) return rc;
-    std::vector<int64_t> cu(n, 0);
-    for (size_t i = 0; i < js.size(); i++) cu[js[i].chain] += (int64_t)counts[i];
+    rc = allreduce_min(ctx, (int32_t *)ctx->jl.p, (size_t)n);     // a7 over int32[n]
+    if (rc) return rc;
     std::vector<int32_t> jstar(n);
     CUDA_TRY(ctx, d2h(ctx, jstar.data(), ctx->jl.p, sizeof(int32_t) * n));
     CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
     for (int i = 0; i < n; i++) fill_infeasible(&out[i], cu[i]);
-    rc = resolve_impl(ctx, cs, cd, disc, jstar, out);
+    if (W == 1 && !ctx->comm) {
+        std::vector<int32_t> all(n, 0);
+        rc = batch_resolve(ctx, cs, cd, disc, jstar, all, 0, out);
+        for (int i = 0; i < n; i++) out[i].cell_updates = cu[i];
+        return rc;
+    }
+    // each winner is re-solved by its owner, then one all-gather of fixed-size records
+    std::vector<int32_t> rowner;
+    resolve_plan(cost, n_c, jstar, W, rowner);
+    int Lmax = 1;
+    for (const auto &c : cs) Lmax = std::max(Lmax, (int)c.c.L);
+    std::vector<int32_t> mine_idx;
+    std::vector<int> per_rank(W, 0);
+    for (int c = 0; c < n; c++) if (rowner[c] >= 0) per_rank[rowner[c]]++;
+    const int slots = std::max(1, *std::max_element(per_rank.begin(), per_rank.end()));
+    const size_t rec = (size_t)kRecHead + 3 * (size_t)Lmax;
+    std::vector<int32_t> st(3 * (size_t)Lmax * n, 0);
+    std::vector<madpipe_alloc> tmp(n);
+    for (int c = 0; c < n; c++) {
+        tmp[c] = out[c];
+        tmp[c].stage_first = st.data() + 3 * (size_t)Lmax * c;
+        tmp[c].stage_last = tmp[c].stage_first + Lmax;
+        tmp[c].stage_proc = tmp[c].stage_last + Lmax;
+    }
+    rc = batch_resolve(ctx, cs, cd, disc, jstar, rowner, R, tmp.data());
+    if (rc) return rc;
+    std::vector<int32_t> sendh((size_t)slots * rec, 0);
+    int k = 0;
+    for (int c = 0; c < n; c++)
+        if (rowner[c] == R) pack_rec(tmp[c], Lmax, sendh.data() + (size_t)(k++) * rec);
+    CUDA_TRY(ctx, ctx->gather.ensure(sizeof(int32_t) * (size_t)slots * rec * (size_t)(W + 1)));
+    int32_t *sendd = (int32_t *)ctx->gather.p, *recvd = sendd + (size_t)slots * rec;
+    CUDA_TRY(ctx, h2d(ctx, sendd, sendh.data(), sizeof(int32_t) * sendh.size()));
+    {
+        std::string why;
+        if (comm_allgather_i32(ctx->comm, sendd, recvd, (size_t)slots * rec, ctx->stream, &why))
+            return fail(ctx, MADPIPE_ENCCL, "%s", why.c_str());
+    }
+    std::vector<int32_t> recvh((size_t)W * slots * rec);
+    CUDA_TRY(ctx, d2h(ctx, recvh.data(), recvd, sizeof(int32_t) * recvh.size()));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    std::vector<int> next(W, 0);
+    for (int c = 0; c < n; c++) {
+        const int r = rowner[c];
+        if (r < 0) continue;
+        unpack_rec(recvh.data() + ((size_t)r * slots + (size_t)(next[r]++)) * rec, Lmax, out[c]);
+    }
     for (int i = 0; i < n; i++) out[i].cell_updates = cu[i];
+    return MADPIPE_OK;
+}
+
+extern "C" int madpipe_batch_plan(int32_t n, const madpipe_chain *chains, const int32_t *P, const double *beta,
+                                  const madpipe_disc *disc, int32_t world, int32_t *owner, int64_t *load,
+                                  int64_t *cost) {
+    if (n < 1 || !chains || !P || !beta || !disc || world < 1 || disc->n_periods < 1)
+        return fail(nullptr, MADPIPE_EINVAL, "bad batch plan arguments");
+    std::vector<ChainSpec> cs;
+    for (int i = 0; i < n; i++) {
+        if (chains[i].L < 1 || P[i] < 1 || !chains[i].uF || !chains[i].uB || !chains[i].a)
+            return fail(nullptr, MADPIPE_EINVAL, "chain %d invalid", i);
+        cs.push_back({chains[i], false, P[i], 1, beta[i]});
+    }
+    std::vector<int32_t> own;
+    std::vector<int64_t> ld, cst;
+    batch_plan(cs, disc, world, own, &ld, &cst);
+    if (owner) std::copy(own.begin(), own.end(), owner);
+    if (load) std::copy(ld.begin(), ld.end(), load);
+    if (cost) std::copy(cst.begin(), cst.end(), cost);
+    return MADPIPE_OK;
+}
+
+extern "C" int madpipe_resolve_plan(int32_t n, const madpipe_chain *chains, const int32_t *P, const double *beta,
+                                    const madpipe_disc *disc, const int32_t *j_star, int32_t world,
+                                    int32_t *owner) {
+    if (n < 1 || !chains || !P || !beta || !disc || !j_star || !owner || world < 1)
+        return fail(nullptr, MADPIPE_EINVAL, "bad resolve plan arguments");
+    std::vector<ChainSpec> cs;
+    for (int i = 0; i < n; i++) cs.push_back({chains[i], false, P[i], 1, beta[i]});
+    std::vector<int64_t> cost;
+    batch_costs(cs, disc, cost);
+    std::vector<int32_t> js(j_star, j_star + n), ro;
+    resolve_plan(cost, disc->n_periods, js, world, ro);
+    std::copy(ro.begin(), ro.end(), owner);
+    return MADPIPE_OK;
+}
+
+extern "C" int madpipe_sweep_batch(madpipe_ctx *ctx, int32_t n, const madpipe_chain *chains, const int32_t *P,
+                                   const int64_t *M, const double *beta, const madpipe_disc *disc, int32_t rank,
+                                   int32_t world, int32_t *j_local, int64_t *cell_updates_out) {
+    int rc = begin(ctx);
+    if (rc) return rc;
+    if (world < 1 || rank < 0 || rank >= world || !j_local)
+        return fail(ctx, MADPIPE_EINVAL, "bad rank/world/j_local");
+    std::vector<ChainSpec> cs;
+    rc = prepare_batch(ctx, n, chains, P, M, beta, disc, cs);
+    if (rc) return rc;
+    std::vector<int32_t> owner;
+    if (world > 1) batch_plan(cs, disc, world, owner, nullptr, nullptr);
+    std::vector<ChainDev> cd;
+    rc = upload_chains(ctx, cs, cd);
+    if (rc) return rc;
+    std::vector<int64_t> cu;
+    rc = batch_sweep(ctx, cs, cd, disc, rank, world, owner, cu);
+    if (rc) return rc;
+    CUDA_TRY(ctx, d2h(ctx, j_local, ctx->jl.p, sizeof(int32_t) * n));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    if (cell_updates_out) std::copy(cu.begin(), cu.end(), cell_updates_out);
+    return MADPIPE_OK;
+}
+
+extern "C" int madpipe_resolve_batch(madpipe_ctx *ctx, int32_t n, const madpipe_chain *chains, const int32_t *P,
+                                     const int64_t *M, const double *beta, const madpipe_disc *disc,
+                                     const int32_t *j_star, int32_t rank, int32_t world, madpipe_alloc *out) {
+    int rc = begin(ctx);
+    if (rc) return rc;
+    if (world < 1 || rank < 0 || rank >= world || !j_star || !out)
+        return fail(ctx, MADPIPE_EINVAL, "bad rank/world/j_star/out");
+    std::vector<ChainSpec> cs;
+    rc = prepare_batch(ctx, n, chains, P, M, beta, disc, cs);
+    if (rc) return rc;
+    std::vector<int32_t> js(j_star, j_star + n), rowner;
+    for (int c = 0; c < n; c++)
+        if (js[c] != INT32_MAX && (js[c] < 0 || js[c] >= disc->n_periods))
+            return fail(ctx, MADPIPE_EINVAL, "j_star[%d] out of range", c);
+    std::vector<int64_t> cost;
+    batch_costs(cs, disc, cost);
+    resolve_plan(cost, disc->n_periods, js, world, rowner);
+    std::vector<ChainDev> cd;
+    rc = upload_chains(ctx, cs, cd);
+    if (rc) return rc;
+    for (int c = 0; c < n; c++) {
+        if (rowner[c] != rank) continue;
+        const int64_t keep = out[c].cell_updates;
+        fill_infeasible(&out[c], keep);
+    }
+    rc = batch_resolve(ctx, cs, cd, disc, js, rowner, rank, out);
     return rc;
 }
 

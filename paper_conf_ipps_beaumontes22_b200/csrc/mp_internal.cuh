@@ -5,6 +5,7 @@
 // readings listed in DESIGN.md section 3.
 #pragma once
 #include <cstdint>
+#include <string>
 #include <cuda_runtime.h>
 
 namespace mp {
@@ -87,9 +88,6 @@ void launch_jobs_init(Job *jobs, int n_jobs, cudaStream_t s);
 void launch_init_slab0(const Job *jobs, int n_jobs, int nmp, int max_cells, cudaStream_t s);
 void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp,
                  cudaStream_t s);
-void launch_step_tma(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int smem,
-                     cudaStream_t s);
-int tma_smem_bytes(int vb, int np, int nmp);
 void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np,
                          int vb, int nsg, int grid, unsigned long long *prof, int n_prod, int tile_block,
                          size_t buf_off, cudaStream_t s);
@@ -97,7 +95,7 @@ void pair_geom(int P, int n_v, int *np, int *n_ptiles, int *n_vtiles, int *n_til
 int pair_list_cap(int max_L);
 size_t pair_entry_bytes();
 int pair_nsl(int np, int nmp);
-bool pair_supported(int P, int nmp, int n_v);
+bool pair_supported(int P, int nmp, int n_v, int max_L);
 void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int fix_slab,
                        cudaStream_t s);
 void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, cudaStream_t s);
@@ -107,7 +105,6 @@ int pair_blocks_per_sm(int nmp, int np, int nsl);
 int persist_blocks_per_sm(int nmp, int np, int vb, int nsg, int n_prod);
 void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
 int persist_nsg(int np, int vb, int nmp);
-void tma_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);
 void launch_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int verify_last,
                   cudaStream_t s);
 void launch_window(const Job *jobs, int n_jobs, int max_L, cudaStream_t s);
@@ -126,5 +123,15 @@ void launch_argmin(const Job *job, int nmp, int32_t *arg_out, int L, int P, int 
                    cudaStream_t s);
 void launch_export(const Job *job, int nmp, double *A_out, int L, int P, int n_v, int n_m,
                    cudaStream_t s);
+
+// ctx-owned NCCL communicator (mp_comm.cu; NCCL is dlopen'ed on first use).
+// Each returns 0 or -1 with *why set.
+int comm_unique_id(uint8_t id[128], std::string *why);
+int comm_init(void **comm, int world, int rank, const uint8_t id[128], std::string *why);
+void comm_destroy(void *comm);
+int comm_allreduce_min_i32(void *comm, int32_t *buf, size_t n, cudaStream_t s, std::string *why);
+int comm_allgather_i32(void *comm, const int32_t *send, int32_t *recv, size_t n_per_rank, cudaStream_t s,
+                       std::string *why);
+int comm_version();
 
 }  // namespace mp

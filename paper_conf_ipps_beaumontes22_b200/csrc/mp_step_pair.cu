@@ -744,7 +744,7 @@ __device__ __forceinline__ void pair_fixup_body(const Job &J, int v, int lane, i
     // The row already holds the clamped min of the other options (values <= tau or
     // +inf); a cell is written back only when option k = l1 lowers it.  FB cells per
     // lane are loaded before any is stored (slab l1-1 is read-only here), so each warp
-    // keeps 3 FB loads in flight.
+    // keeps FB loads in flight.
 #ifndef MP_FIX_FB
 #define MP_FIX_FB 4
 #endif
@@ -807,7 +807,10 @@ int pair_nsl(int np, int nmp) {
     return slots - slots % kPairProd;                       // split evenly between the producers
 }
 
-bool pair_supported(int P, int nmp, int n_v) { return P >= 2 && (nmp == 4 || nmp == 8) && n_v <= 65535; }
+// key = (k << 16) | v' (pair_trans_kernel) and PairEntry.k are 16-bit in k: layers < 32768
+bool pair_supported(int P, int nmp, int n_v, int max_L) {
+    return P >= 2 && (nmp == 4 || nmp == 8) && n_v <= 65535 && max_L < 32768;
+}
 
 void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int fix_slab,
                        cudaStream_t s) {

@@ -1,43 +1,31 @@
-"""Multi-GPU controller: one process per GPU.
+"""Multi-GPU bootstrap: one process per GPU.
 
-Candidate periods are independent units, sharded interleaved (rank r owns
-j = r, r+W, ...; the cost of a candidate grows with its period, so interleaving
-balances the ranks).  Each rank sweeps its shard (madpipe_sweep), the ranks
-min-reduce their smallest feasible candidate index with ONE all-reduce (the
-path's only exchange step, a7: 4 bytes over NVLink with NCCL), and every rank
-re-solves the winner and traces it back (madpipe_resolve) -- deterministic,
-so no broadcast of the allocation is needed.
-
-The same function runs on CPU process groups (gloo) in the tests, with the two
-library calls replaced by test doubles (``sweep_fn`` / ``resolve_fn``).
+The path's only exchange step -- a7, the MIN all-reduce of the ranks' smallest
+feasible candidate indices (and, for a batch, the all-gather of the winners'
+allocations) -- runs inside libmadpipe over the ctx's own NCCL communicator
+(madpipe_ctx_create with rank, world and an NCCL id).  So an N-GPU solve is one
+C call per rank: ``context(...).solve_dev(...)``.  This module only does the
+process bootstrap: rank 0 creates the 128-byte NCCL id (madpipe_get_unique_id)
+and the launcher's process group (torch.distributed, any backend) carries it to
+the other ranks.  Nothing here touches the DP's data.
 """
 from __future__ import annotations
 
-import torch
 import torch.distributed as dist
 
-INT32_MAX = 2 ** 31 - 1
+from . import Context, get_unique_id
 
 
-def solve_distributed(chain, P, M, beta, n_mem, n_delay, n_periods, v_range=0, early_exit=False,
-                      ctx=None, group=None, device=None, sweep_fn=None, resolve_fn=None):
-    """Returns (result dict, this rank's cell-update count)."""
-    rank = dist.get_rank(group)
-    world = dist.get_world_size(group)
-    if device is None:
-        device = torch.device("cuda", torch.cuda.current_device())
-    jl = torch.full((1,), INT32_MAX, dtype=torch.int32, device=device)
-    if sweep_fn is None:
-        cu = ctx.sweep(chain, P, M, beta, n_mem, n_delay, n_periods, rank, world, jl.data_ptr(),
-                       v_range=v_range, early_exit=early_exit)
-    else:
-        cu = sweep_fn(rank, world, jl)
-    dist.all_reduce(jl, op=dist.ReduceOp.MIN, group=group)        # a7
-    if jl.is_cuda:
-        torch.cuda.current_stream(jl.device).synchronize()
-    if resolve_fn is None:
-        res = ctx.resolve(chain, P, M, beta, n_mem, n_delay, n_periods, jl.data_ptr(),
-                          v_range=v_range)
-    else:
-        res = resolve_fn(jl)
-    return res, cu
+def share_id(group=None) -> bytes:
+    """Rank 0's NCCL id, broadcast over the torch process group (bootstrap only)."""
+    obj = [get_unique_id() if dist.get_rank(group) == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    return obj[0]
+
+
+def context(device: int, stream=None, group=None, mem_budget: int = 0) -> Context:
+    """A Context that is rank ``dist.get_rank(group)`` of ``dist.get_world_size(group)``
+    with a communicator over all of them (also at world 1)."""
+    nid = share_id(group)
+    return Context(device, stream=stream, mem_budget=mem_budget, rank=dist.get_rank(group),
+                   world=dist.get_world_size(group), nccl_id=nid)

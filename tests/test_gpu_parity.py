@@ -39,7 +39,7 @@ def _ctx_with_kernel(kernel):
             os.environ["MADPIPE_KERNEL"] = old
 
 
-@pytest.fixture(scope="module", params=["pair", "persist", "v1", "tma"])
+@pytest.fixture(scope="module", params=["pair", "persist", "v1"])
 def kctx(request):
     c = _ctx_with_kernel(request.param)
     yield c
@@ -250,7 +250,7 @@ def test_geometry_extremes(P, n_m, n_v, L):
     M = int((3 * ch["W"].sum() + 3 * ch["a"].sum()) * 0.6) + 1
     n_c = 9
     ref = oracle.solve(ch, P, M, 25.0, n_m, n_v, n_c, v_range=1, n_threads=4)
-    for kernel in ("pair", "persist", "v1", "tma"):
+    for kernel in ("pair", "persist", "v1"):
         c = _ctx_with_kernel(kernel)
         try:
             tau, root = c.candidates(ch, P, M, 25.0, n_m, n_v, n_c, v_range=1)
@@ -336,3 +336,88 @@ def test_work_counters_agree_across_kernels():
         assert got["useful_updates"] <= got["effective_updates"], (kernel, got)
         if kernel != "v1":
             assert got["useful_updates"] > 0, (kernel, got)
+
+
+# ---------------------------------------------------------------- communication-bound chains
+def _comm_cases(n, seed):
+    """Activations up to 400 bytes, beta in [5, 30] (C(i) = 2 a_i / beta far above the
+    stage loads) and a candidate grid dense near lb: C(k-1) > tau prunes splits
+     and links bound the allocation period."""
+    rng = np.random.default_rng(seed)
+    for i in range(n):
+        L = int(rng.integers(4, 20))
+        P = int(rng.choice([2, 3, 5, 9, 34, 40, 70]))
+        ch = chaingen.tiny(rng, L, a_hi=400)
+        n_m = int(rng.choice([3, 4, 5, 8]))
+        n_v = int(rng.choice([5, 16, 51]))
+        vr = int(rng.integers(0, 2))
+        mem = 3 * int(ch["W"].sum()) + 3 * int(ch["a"].sum()) + 1
+        M = int(mem * rng.uniform(0.15, 0.9)) + 1
+        beta = float(rng.uniform(5.0, 30.0))
+        yield ch, P, M, beta, n_m, n_v, 24, vr
+
+
+def test_comm_heavy_every_kernel(kctx):
+    ctx = kctx
+    pairs = with_c = 0
+    for ch, P, M, beta, n_m, n_v, n_c, vr in _comm_cases(40, 91):
+        ref = oracle.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr, n_threads=4)
+        tau, root = ctx.candidates(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
+        assert np.array_equal(tau, ref["tau"]) and np.array_equal(root, ref["root"]), (P, n_m, n_v, vr)
+        got = ctx.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
+        _same_solution(got, ref)
+        j = max(ref["cand_index"], 0)
+        A, ARG = ctx.dp_table(ch, P, M, beta, n_m, n_v, n_c, j=j, v_range=vr)
+        A_ref, ARG_ref, _ = oracle.table(ch, P, M, beta, n_m, n_v, vr, ref["tau"][j])
+        assert np.array_equal(A, A_ref) and np.array_equal(ARG, ARG_ref)
+        _verify(ch, P, M, beta, got)
+        cmax = max(2.0 * ch["a"][i] / beta for i in range(1, len(ch["uF"]))) if len(ch["uF"]) > 1 else 0.0
+        pairs += n_c
+        with_c += int(sum(cmax > t for t in tau))
+    assert with_c >= 0.3 * pairs, (with_c, pairs)
+
+
+# ---------------------------------------------------------------- GPT: stratified high periods
+def test_gpt_stratified_candidates_and_slabs(ctx):
+    """SURVEY.md 8(d)'s GPT sample (j <= j*, j*+1..8, 16 stratified above, 511/767/1023)
+    at full size: every candidate's root, and two whole table slabs (l = L/2, l = L) of
+    each sampled candidate, against values written by scripts/oracle_gpt_samples.py."""
+    import hashlib
+    cfg = configs.load("gpt")
+    sam = configs.load("gpt_oracle_samples")
+    assert sam["digest"] == cfg["digest"]
+    ch = chaingen.make(cfg["chain"])
+    a = _args(cfg)
+    tau, root = ctx.candidates(ch, *a)
+    L = cfg["L"]
+    assert len(sam["samples"]) >= 30
+    for s in sam["samples"]:
+        j = s["j"]
+        assert tau[j] == float.fromhex(s["tau"]), j
+        assert root[j] == float.fromhex(s["root"]), j
+        A, _ = ctx.dp_table(ch, *a, j=j, with_arg=False)
+        for l, dg in s["slab_sha256"].items():
+            assert hashlib.sha256(np.ascontiguousarray(A[int(l)]).tobytes()).hexdigest() == dg, (j, l)
+    assert max(s["j"] for s in sam["samples"]) == cfg["n_periods"] - 1
+
+
+def test_solve_dev_equals_solve_equals_oracle(ctx):
+    """madpipe_solve_dev (the entry bench.py times) on device-resident chains gives the
+    same result as madpipe_solve on host arrays, and as the oracle."""
+    import torch
+    for name in ("gpt", "resnet50"):
+        cfg = configs.load(name)
+        ch = chaingen.make(cfg["chain"])
+        a = _args(cfg)
+        d = {k: torch.from_numpy(np.ascontiguousarray(ch[k])).cuda() for k in ("uF", "uB", "W", "a")}
+        dev = ctx.solve_dev(d, *a)
+        host = ctx.solve(ch, *a)
+        _same_solution(dev, host)
+        assert dev["cell_updates"] == host["cell_updates"]
+        assert dev["cand_index"] == cfg["oracle_cand_index"]
+        ref = oracle.solve(ch, *a, early_exit=True, n_threads=8)
+        _same_solution(dev, ref)
+    for ch, P, M, beta, n_m, n_v, n_c, vr in _fuzz_cases(10, 31):
+        d = {k: torch.from_numpy(np.ascontiguousarray(ch[k])).cuda() for k in ("uF", "uB", "W", "a")}
+        ref = oracle.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
+        _same_solution(ctx.solve_dev(d, P, M, beta, n_m, n_v, n_c, v_range=vr), ref)

@@ -116,3 +116,60 @@ def test_product_never_imports_oracle():
                 src = open(os.path.join(dirpath, f)).read()
                 assert not re.search(r"^\s*(import|from)\s+oracle", src, re.M), f
                 assert "madpipe_oracle" not in src, f
+
+
+def _plan_batch(seed, n=12):
+    rng = np.random.default_rng(seed)
+    chains = [chaingen.tiny(rng, int(rng.integers(2, 40))) for _ in range(n)]
+    Ps = [int(rng.integers(1, 9)) for _ in range(n)]
+    betas = [float(rng.uniform(5, 50)) for _ in range(n)]
+    return chains, Ps, betas
+
+
+def test_batch_plan_lpt():
+    """madpipe_batch_plan: every (chain, candidate) pair has exactly one
+    owner, the cost of a pair is its exact cell-update count plus the fixed row work,
+    the plan is deterministic, and LPT keeps the ranks within one largest job."""
+    chains, Ps, betas = _plan_batch(5)
+    n_m, n_v, n_c = 4, 8, 16
+    for world in (1, 2, 3, 8):
+        owner, load, cost = mp.batch_plan(chains, Ps, betas, n_m, n_v, n_c, world)
+        owner2, load2, _ = mp.batch_plan(chains, Ps, betas, n_m, n_v, n_c, world)
+        assert np.array_equal(owner, owner2) and np.array_equal(load, load2)
+        assert owner.min() >= 0 and owner.max() < world
+        for r in range(world):
+            assert load[r] == cost[owner == r].sum()
+        assert load.sum() == cost.sum()
+        assert load.max() - load.min() <= cost.max()
+    for c, (ch, P, b) in enumerate(zip(chains, Ps, betas)):
+        pre = oracle.prep(ch, P, b)
+        for j in (0, 7, 15):
+            tau = pre["lb"] + j * ((pre["ub"] - pre["lb"]) / (n_c - 1))
+            L = len(ch["uF"])
+            assert cost[c, j] == mp.cell_updates(ch, P, n_m, n_v, tau) + (L + 1) * n_v * P
+
+
+def test_resolve_plan_one_owner_per_winner():
+    chains, Ps, betas = _plan_batch(6)
+    jstar = np.array([c % 16 if c % 3 else 2 ** 31 - 1 for c in range(len(chains))], np.int32)
+    for world in (1, 2, 5):
+        own = mp.resolve_plan(chains, Ps, betas, 4, 8, 16, jstar, world)
+        for c in range(len(chains)):
+            if jstar[c] == 2 ** 31 - 1:
+                assert own[c] == -1
+            else:
+                assert 0 <= own[c] < world
+
+
+def test_nccl_unique_id_on_cpu():
+    """madpipe_get_unique_id needs only libnccl (dlopen'ed), not a GPU."""
+    a = mp.get_unique_id()
+    b = mp.get_unique_id()
+    assert len(a) == 128 and a != b
+
+
+def test_ctx_create_rejects_bad_rank_world():
+    for rank, world, nid in [(0, 0, None), (2, 2, b"\0" * 128), (-1, 2, b"\0" * 128), (1, 2, None)]:
+        with pytest.raises(mp.MadpipeError) as e:
+            mp.Context(0, rank=rank, world=world, nccl_id=nid)
+        assert e.value.rc == N.EINVAL
