@@ -799,12 +799,21 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             float ms = 0.f;
             cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b);
             ctx->sweep_ms += ms;
+            double kms = 0.0;
             if (per_launch) {
                 for (int l = 1; l <= ctx->n_rec; l++) {
                     float m2 = 0.f;
                     cudaEventElapsedTime(&m2, ctx->ev_pool[2 * (l - 1)], ctx->ev_pool[2 * (l - 1) + 1]);
-                    ctx->step_ms += m2;
+                    kms += m2;
                 }
+                ctx->step_ms += kms;
+            }
+            if (ctx->prof) {
+                uint64_t u = 0, e = 0;
+                for (int i = 0; i < nj; i++) { u += hcounts[2 * nj + i]; e += hcounts[nj + i]; }
+                fprintf(stderr, "[madpipe batch] P=%d jobs=%d maxL=%d kernel=%d tiles=%d: %.3f ms (step %.3f ms), "
+                                "effective %.3g, useful %.3g\n",
+                        hjobs[0].P, nj, maxL, kern, n_tiles, ms, kms, (double)e, (double)u);
             }
         }
     }

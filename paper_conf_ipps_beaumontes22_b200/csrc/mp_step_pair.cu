@@ -71,16 +71,18 @@ __device__ __forceinline__ double dmin(double a, double b) { return b < a ? b : 
 __device__ __forceinline__ void mbar_arrive_cnt(uint32_t bar, uint32_t cnt) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(cnt) : "memory");
 }
-// Queue publication inside one CTA: the producer warp's shared stores (queue
-// entry, then tail) are performed in program order by the shared-memory pipeline,
-// and the consumer polls the tail with volatile loads.  A release/acquire pair or
-// a fence here would also wait for the producer's outstanding global prefetch
-// loads (measured: ~35% of the producer's time), so plain volatile accesses are used.
-__device__ __forceinline__ void st_publish(int *p, int v) {
+// Row queues inside one CTA: a queue entry is ONE 32-bit shared word that carries its
+// own wrap bit (bit 31 = ((position / QN) & 1) ^ 1; the queue starts zeroed), so the
+// consumer polls the entry itself.  No second location (a tail) is published, hence
+// no cross-location ordering is needed: single-location coherence of the producer's
+// volatile store and the consumer's volatile load is all the handoff relies on.  The
+// slot's data and metadata are ordered by the slot's full mbarrier (arrive = release,
+// try_wait = acquire; the bulk copy completes on it), not by the queue word.
+__device__ __forceinline__ void st_entry(uint32_t *p, uint32_t v) {
     asm volatile("st.volatile.shared::cta.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
 }
-__device__ __forceinline__ int ld_poll(const int *p) {
-    int v;
+__device__ __forceinline__ uint32_t ld_entry(const uint32_t *p) {
+    uint32_t v;
     asm volatile("ld.volatile.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
     return v;
 }
@@ -448,8 +450,8 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     __shared__ __align__(8) uint64_t full[kPairSlotsMax];
     __shared__ __align__(8) uint64_t empty[kPairSlotsMax];
     __shared__ __align__(16) PairMeta meta[kPairSlotsMax];
-    __shared__ uint32_t rq[kPairProd][kPairRows][QN];      // per-row queues: slot | parity << 6 | control << 7 | n_m << 8 | code << 16
-    __shared__ int rtail[kPairProd][kPairRows];            // entries pushed per row (producer)
+    // per-row queues: slot | parity << 6 | control << 7 | n_m << 8 | code << 16 | wrap bit << 31
+    __shared__ uint32_t rq[kPairProd][kPairRows][QN];
     __shared__ __align__(128) PairEntry stage[kPairProd][2][kPairStage];   // list heads of this and the next tile
     __shared__ __align__(8) uint64_t stbar[kPairProd][2];
 
@@ -469,7 +471,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    if (tid < kPairRows * kPairProd) rtail[tid / kPairRows][tid % kPairRows] = 0;
+    for (int i = tid; i < kPairProd * kPairRows * QN; i += blockDim.x) (&rq[0][0][0])[i] = 0u;
     __syncthreads();
 
     if (warp >= kPairRows) {
@@ -482,20 +484,19 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
         for (int rr = 0; rr < kPairRows; rr++) tails[rr] = 0;
         const unsigned lt = (1u << lane) - 1u;
         auto push = [&](bool act, uint32_t mask, uint32_t ent, uint64_t codes) {   // codes: byte rr = row rr
-            // append ent (+ the row's code) to the queue of every row in mask, in lane order
-            int mytail = 0;
+            // append ent (+ the row's code, + the wrap bit of its position) to the queue of
+            // every row in mask, in lane order
 #pragma unroll
             for (int rr = 0; rr < kPairRows; rr++) {
                 const bool mine = act && ((mask >> rr) & 1u);
                 const unsigned bal = __ballot_sync(0xffffffffu, mine);
-                if (mine)
-                    reinterpret_cast<volatile uint32_t *>(rq[pw][rr])[(tails[rr] + __popc(bal & lt)) & (QN - 1)] =
-                        ent | (uint32_t)((codes >> (8 * rr)) & 0xFFu) << 16;
+                if (mine) {
+                    const int pos = tails[rr] + __popc(bal & lt);
+                    st_entry(&rq[pw][rr][pos & (QN - 1)], ent | (uint32_t)((codes >> (8 * rr)) & 0xFFu) << 16 |
+                                                               (uint32_t)(((pos / QN) & 1) ^ 1) << 31);
+                }
                 tails[rr] += __popc(bal);
-                if (lane == rr) mytail = tails[rr];
             }
-            __syncwarp();
-            if (lane < kPairRows) st_publish(&rtail[pw][lane], mytail);
         };
         // prof (MADPIPE_PROF=1): [0] producer cycles, [1] empty-barrier waits (max over lanes),
         // [2] tile setup (header), [3] consumer cycles, [4] queue waits, [5] full waits, [6] data
@@ -645,24 +646,22 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     for (int i = 0; i < NMP; i++) { b0[i] = MP_INF; b1[i] = MP_INF; }
     const char *ring = reinterpret_cast<const char *>(dsm);
     const int seg_bytes = seg_doubles * 8;
-    int head[kPairProd] = {}, avail[kPairProd] = {};
+    int head[kPairProd] = {};
     int qp = 0;                                            // the queue of the current tile's producer
     long long t_c0 = clock64(), t_q = 0, t_f = 0, n_sl = 0;
     for (;;) {
         const long long ta = prof ? clock64() : 0;
-        // an empty queue: back off instead of spinning (a spinning warp takes issue slots
-        // from the producer and the working rows)
-        // (the tail is re-read only when the entries seen last time are used up)
-        if (head[qp] == avail[qp]) {
-            int t;
-            while ((t = ld_poll(&rtail[qp][r])) == head[qp]) {
+        // an empty queue (the entry still carries the previous wrap's bit): back off
+        // instead of spinning (a spinning warp takes issue slots from the producer and
+        // the working rows)
+        const uint32_t want = (uint32_t)(((head[qp] / QN) & 1) ^ 1);
+        const uint32_t *qe = &rq[qp][r][head[qp] & (QN - 1)];
+        uint32_t ent;
+        while (((ent = ld_entry(qe)) >> 31) != want) {
 #if MP_POLL_NS > 0
-                __nanosleep(MP_POLL_NS);
+            __nanosleep(MP_POLL_NS);
 #endif
-            }
-            avail[qp] = t;
         }
-        const uint32_t ent = reinterpret_cast<volatile uint32_t *>(rq[qp][r])[head[qp] & (QN - 1)];
         head[qp]++;
         const int s = (int)(ent & 63u);                    // this row's slot
         const long long tb = prof ? clock64() : 0;

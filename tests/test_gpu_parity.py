@@ -340,14 +340,18 @@ def test_work_counters_agree_across_kernels():
 
 # ---------------------------------------------------------------- communication-bound chains
 def _comm_cases(n, seed):
-    """Activations up to 400 bytes, beta in [5, 30] (C(i) = 2 a_i / beta far above the
-    stage loads) and a candidate grid dense near lb: C(k-1) > tau prunes splits
-     and links bound the allocation period."""
+    """Two boundaries with activations of 200-400 bytes and beta in [5, 30] (C(i) =
+    2 a_i / beta far above the stage loads, while sum C stays small enough that the
+    uniform candidate grid on [lb, ub] spends about a third of its periods below
+    max C): C(k-1) > tau prunes splits and links bound the allocation
+    period (P:153)."""
     rng = np.random.default_rng(seed)
     for i in range(n):
         L = int(rng.integers(4, 20))
         P = int(rng.choice([2, 3, 5, 9, 34, 40, 70]))
-        ch = chaingen.tiny(rng, L, a_hi=400)
+        ch = chaingen.tiny(rng, L)
+        hv = rng.choice(np.arange(1, L), size=min(2, L - 1), replace=False)
+        ch["a"][hv] = rng.integers(200, 400, size=len(hv))
         n_m = int(rng.choice([3, 4, 5, 8]))
         n_v = int(rng.choice([5, 16, 51]))
         vr = int(rng.integers(0, 2))
@@ -374,7 +378,7 @@ def test_comm_heavy_every_kernel(kctx):
         cmax = max(2.0 * ch["a"][i] / beta for i in range(1, len(ch["uF"]))) if len(ch["uF"]) > 1 else 0.0
         pairs += n_c
         with_c += int(sum(cmax > t for t in tau))
-    assert with_c >= 0.3 * pairs, (with_c, pairs)
+    assert with_c >= 0.25 * pairs, (with_c, pairs)
 
 
 # ---------------------------------------------------------------- GPT: stratified high periods
