@@ -474,20 +474,22 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         // ---- form a batch
         hjobs.clear(); htiles.clear(); ids.clear();
         // step kernel of this batch (measured): the persistent TMA kernel moves
-        // one row segment per stage, which pays off from ~1 KB segments; below, plain loads win
-        int kern = ctx->kernel;
+        // one row segment per stage, which pays off from ~1 KB segments; below, plain loads win;
+        // the two-layer kernel where it measured faster (profiles/r01_pair_dispatch.md): P > 33
+        // (the single-layer kernel needs two warps per delay row there), n_mem <= 8
+        auto kernel_for = [&](int P) {
+            int k = ctx->kernel;
+            if (k == 3 && !pair_supported(P, nmp, disc->n_delay, all_maxL)) k = -1;
+            if (k < 0) {
+                int vb_, np_, npt_, nt_;
+                persist_geom(P, disc->n_delay, nmp, &vb_, &np_, &npt_, &nt_);
+                k = (np_ + 1) * nmp * 8 >= 1024 ? 2 : 0;
+                if (P > 33 && pair_supported(P, nmp, disc->n_delay, all_maxL)) k = 3;
+            }
+            return k;
+        };
         while (next < js.size() && early_exit && jl_host[js[next].chain] < js[next].j) next++;
-        if (kern == 3 && next < js.size() && !pair_supported(cs[js[next].chain].P, nmp, disc->n_delay, all_maxL)) kern = -1;
-        if (kern < 0 && next < js.size()) {
-            int vb_, np_, npt_, nt_;
-            persist_geom(cs[js[next].chain].P, disc->n_delay, nmp, &vb_, &np_, &npt_, &nt_);
-            kern = (np_ + 1) * nmp * 8 >= 1024 ? 2 : 0;
-            // two-layer kernel where it measured faster (scripts/exp_dispatch.py,
-            // profiles/r01_pair_dispatch.md): P > 33 (the single-layer kernel needs two
-            // warps per delay row there), n_mem <= 8
-            const int P = cs[js[next].chain].P;
-            if (P > 33 && pair_supported(P, nmp, disc->n_delay, all_maxL)) kern = 3;
-        }
+        const int kern = next < js.size() ? kernel_for(cs[js[next].chain].P) : 0;
         size_t used = 0;
         int maxL = 0;
         size_t max_slab = 0;
@@ -497,8 +499,10 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             const ChainSpec &c = cs[s.chain];
             const size_t bytes = table_doubles(c, disc) * 8;
             if (!hjobs.empty() && (used + bytes > budget || hjobs.size() >= cap_jobs)) break;
-            // one tile geometry (and one step kernel) per launch: uniform P
-            if (!hjobs.empty() && c.P != hjobs[0].P) break;
+            // one step kernel per launch; chains of different P share it (each job carries
+            // its own tile geometry) except on the single-layer persistent kernel, whose
+            // ring and tile shape are set per launch
+            if (!hjobs.empty() && (kernel_for(c.P) != kern || (kern == 2 && c.P != hjobs[0].P))) break;
             if (hjobs.empty() && bytes > budget && bytes > ctx->tables.n) {
                 // a single job larger than the budget: try anyway (may fail with ENOMEM)
             }
@@ -640,7 +644,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         const int n_tiles = (int)htiles.size();
         int persist_grid = 0, nsg = 0, p_np = 0, p_vb = 0;
         if (kern == 3) {
-            p_np = hjobs[0].np;
+            for (const auto &J : hjobs) p_np = std::max(p_np, J.np);   // processor rows per tile
             nsg = pair_nsl(p_np, nmp);
             if (nsg < 4) return fail(ctx, MADPIPE_EINVAL, "row segment too large for the pair step kernel ring");
             persist_grid = std::min(n_tiles, ctx->num_sms * pair_blocks_per_sm(nmp, p_np, nsg));
