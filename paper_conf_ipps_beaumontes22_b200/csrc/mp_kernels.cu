@@ -458,6 +458,7 @@ __global__ void traceback_kernel(const Job *jobs, int nmp, TraceOut *outs, int32
         const int l = s_l, p = s_p, v = s_v, m = s_m;
         if (l == 0 || s_done) break;
         if (p == 0) {   // base case: stage 1..l on the special GPU
+            __syncthreads();   // every thread has read s_l before thread 0 overwrites it (p is block-uniform)
             if (threadIdx.x == 0) {
                 first[s_ns] = 1; last[s_ns] = l; proc[s_ns] = -1; s_ns++;
                 s_l = 0;

@@ -190,6 +190,7 @@ __global__ void lit_traceback_kernel(const Job *job, LitGeom G, int nmp, int32_t
         const int l = s_l, p = s_p, t = s_t, v = s_v, m = s_m;
         if (l == 0 || s_done) break;
         if (p == 0) {
+            __syncthreads();   // every thread has read s_l before thread 0 overwrites it (p is block-uniform)
             if (threadIdx.x == 0) { first[s_ns] = 1; last[s_ns] = l; kind[s_ns] = 1; s_ns++; s_l = 0; }
             continue;
         }

@@ -78,12 +78,25 @@ __device__ __forceinline__ void mbar_arrive_cnt(uint32_t bar, uint32_t cnt) {
 // volatile store and the consumer's volatile load is all the handoff relies on.  The
 // slot's data and metadata are ordered by the slot's full mbarrier (arrive = release,
 // try_wait = acquire; the bulk copy completes on it), not by the queue word.
+// MP_QUEUE_ATOMIC=1: the same handoff through shared-memory atomics (exchange / or 0),
+// which compute-sanitizer racecheck recognises as synchronising (A/B variant).
+#ifndef MP_QUEUE_ATOMIC
+#define MP_QUEUE_ATOMIC 0
+#endif
 __device__ __forceinline__ void st_entry(uint32_t *p, uint32_t v) {
+#if MP_QUEUE_ATOMIC
+    asm volatile("atom.shared::cta.exch.b32 _, [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+#else
     asm volatile("st.volatile.shared::cta.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+#endif
 }
 __device__ __forceinline__ uint32_t ld_entry(const uint32_t *p) {
     uint32_t v;
+#if MP_QUEUE_ATOMIC
+    asm volatile("atom.shared::cta.or.b32 %0, [%1], 0;" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+#else
     asm volatile("ld.volatile.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+#endif
     return v;
 }
 
