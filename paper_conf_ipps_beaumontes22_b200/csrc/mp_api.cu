@@ -17,6 +17,7 @@
 #include <vector>
 
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include "../../include/madpipe.h"
 #include "mp_internal.cuh"
@@ -76,6 +77,14 @@ struct madpipe_ctx {
 };
 
 static thread_local std::string g_err;
+
+// NVTX ranges per phase of the path (a1 prep, a2-a6 sweep batches, a7 all-reduce, a8 resolve
+// + traceback, batch plan / all-gather): header-only NVTX v3, a no-op unless a tool
+// (nsys, ncu --nvtx) attaches.
+struct Nvtx {
+    explicit Nvtx(const char *name) { nvtxRangePushA(name); }
+    ~Nvtx() { nvtxRangePop(); }
+};
 
 static int fail(madpipe_ctx *ctx, int code, const char *fmt, ...) {
     char buf[512];
@@ -374,6 +383,7 @@ struct JobSpec {
 
 // Upload chains (if on host), allocate derived arrays, run prep_kernel.
 int upload_chains(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, std::vector<ChainDev> &cd) {
+    Nvtx nv("madpipe a1 prep");
     const int n = (int)cs.size();
     size_t bytes = 0;
     auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
@@ -533,6 +543,10 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             ids.push_back((int)next);
         }
         if (hjobs.empty()) break;
+        char nv_name[96];
+        snprintf(nv_name, sizeof nv_name, "madpipe a2-a6 batch: %d jobs, P=%d, kernel %d", (int)hjobs.size(),
+                 hjobs[0].P, kern);
+        Nvtx nv(nv_name);
         if (cap_jobs != SIZE_MAX) cap_jobs *= 2;
         CUDA_TRY(ctx, ctx->tables.ensure(used));
         for (auto &J : hjobs) J.table = (double *)((char *)ctx->tables.p + (uintptr_t)J.table);
@@ -867,6 +881,7 @@ void fill_infeasible(madpipe_alloc *out, int64_t cu) {
 // Resolve the winners (one job per chain with jstar[c] != INT32_MAX).
 int resolve_impl(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vector<ChainDev> &cd,
                  const madpipe_disc *disc, const std::vector<int32_t> &jstar, madpipe_alloc *outs) {
+    Nvtx nv("madpipe a8 resolve + traceback");
     std::vector<JobSpec> js;
     int maxL = 1;
     for (int c = 0; c < (int)cs.size(); c++) {
@@ -946,6 +961,7 @@ std::vector<JobSpec> shard_jobs(int chain, int n_c, int rank, int world) {
 // the ctx's stream.  Without a communicator (world 1) this is the identity.
 int allreduce_min(madpipe_ctx *ctx, int32_t *dev, size_t n) {
     if (!ctx->comm) return MADPIPE_OK;
+    Nvtx nv("madpipe a7 allreduce(MIN)");
     std::string why;
     if (comm_allreduce_min_i32(ctx->comm, dev, n, ctx->stream, &why))
         return fail(ctx, MADPIPE_ENCCL, "%s", why.c_str());
@@ -1086,6 +1102,7 @@ void lpt(const std::vector<int64_t> &cost, const std::vector<int32_t> &items, in
 // owner[c * n_c + j] = rank that evaluates candidate j of chain c
 void batch_plan(const std::vector<ChainSpec> &cs, const madpipe_disc *disc, int world, std::vector<int32_t> &owner,
                 std::vector<int64_t> *load, std::vector<int64_t> *cost_out) {
+    Nvtx nv("madpipe batch plan (LPT)");
     std::vector<int64_t> cost;
     batch_costs(cs, disc, cost);
     owner.assign(cost.size(), 0);
@@ -1320,6 +1337,7 @@ extern "C" int madpipe_solve_batch(madpipe_ctx *ctx, int32_t n, const madpipe_ch
     int32_t *sendd = (int32_t *)ctx->gather.p, *recvd = sendd + (size_t)slots * rec;
     CUDA_TRY(ctx, h2d(ctx, sendd, sendh.data(), sizeof(int32_t) * sendh.size()));
     {
+        Nvtx nv("madpipe batch allgather");
         std::string why;
         if (comm_allgather_i32(ctx->comm, sendd, recvd, (size_t)slots * rec, ctx->stream, &why))
             return fail(ctx, MADPIPE_ENCCL, "%s", why.c_str());

@@ -110,7 +110,7 @@ constexpr int kPairRows = 2 * kPairVB;           // output rows (= consumer warp
 constexpr int kPairE = 16 / kPairVB;             // extra v-tiles: layer l+1 rows are shifted by <= 16 levels
 constexpr int kPairCtas = 8 / kPairVB;           // resident CTAs per SM (one producer warp each)
 constexpr int kPairNp = 64;                      // processor rows per tile (2 per consumer thread)
-constexpr int kPairSlotsMax = 32;
+constexpr int kPairSlotsMax = kPairVB > 4 ? 48 : 32;  // ring slots (6-bit slot index in the queue word)
 #ifndef MP_PAIR_NPROD
 #define MP_PAIR_NPROD 1
 #endif
@@ -133,12 +133,12 @@ constexpr int kPairStage = MP_PAIR_STAGE;        // list head (header + entries)
 struct PairEntry {
     uint16_t k;        // option k: the source is slab k-1
     uint16_t vp;       // next delay level v' (source row)
-    uint8_t mask;      // output rows of the tile that read it (bit r: r < 4 layer l, else l+1)
-    uint8_t pad[3];
-    uint8_t code[8];   // per row r < kPairRows: d (bits 0-6, clamped to 127) | nf << 7
+    uint16_t mask;     // output rows of the tile that read it (bit r: r < kPairVB layer l, else l+1)
+    uint16_t pad;
+    uint8_t code[kPairRows];   // per row r: d (bits 0-6, clamped to 127) | nf << 7
     double U0, U1;     // U(k,l), U(k,l+1)
 };
-static_assert(sizeof(PairEntry) == 32, "PairEntry size");
+static_assert(sizeof(PairEntry) == 24 + kPairRows, "PairEntry size");
 
 // Tile header (the first kPairHdr entries of a tile list): what the producer
 // needs for the tile without reading the job descriptor.  n < 0: the job has no
@@ -153,7 +153,7 @@ struct PairHdr {
     uint32_t *flA;     // rowflag + l * n_v
     int32_t n_v, P;
     int32_t v0A, v0B;  // first delay row of layer l / layer l+1 in the tile
-    int64_t pad_;
+    int64_t pad_[1 + (kPairHdr * (24 + kPairRows) - 64) / 8];
 };
 static_assert(sizeof(PairHdr) == kPairHdr * sizeof(PairEntry), "PairHdr size");
 
@@ -307,7 +307,7 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
         hd.P = J.P;
         hd.v0A = vt * kPairVB;
         hd.v0B = vt * kPairVB - delta;
-        hd.pad_ = 0;
+        for (auto &x : hd.pad_) x = 0;
         *reinterpret_cast<PairHdr *>(tl) = hd;
     }
     for (int o = 16; o > 0; o >>= 1) {
@@ -458,7 +458,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     prof = nullptr;                                        // cycle counters compiled out (MADPIPE_PROF reads zeros)
 #endif
     constexpr int C = NMP / 2;
-    constexpr int QN = 32;                                 // queue entries per row (>= slots)
+    constexpr int QN = kPairSlotsMax > 32 ? 64 : 32;       // queue entries per row (>= slots, power of 2)
     extern __shared__ __align__(128) unsigned char dsm[];
     __shared__ __align__(8) uint64_t full[kPairSlotsMax];
     __shared__ __align__(8) uint64_t empty[kPairSlotsMax];
@@ -496,7 +496,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
 #pragma unroll
         for (int rr = 0; rr < kPairRows; rr++) tails[rr] = 0;
         const unsigned lt = (1u << lane) - 1u;
-        auto push = [&](bool act, uint32_t mask, uint32_t ent, uint64_t codes) {   // codes: byte rr = row rr
+        auto push = [&](bool act, uint32_t mask, uint32_t ent, uint64_t codes, uint64_t codes_hi) {   // byte rr = row rr
             // append ent (+ the row's code, + the wrap bit of its position) to the queue of
             // every row in mask, in lane order
 #pragma unroll
@@ -505,7 +505,8 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 const unsigned bal = __ballot_sync(0xffffffffu, mine);
                 if (mine) {
                     const int pos = tails[rr] + __popc(bal & lt);
-                    st_entry(&rq[pw][rr][pos & (QN - 1)], ent | (uint32_t)((codes >> (8 * rr)) & 0xFFu) << 16 |
+                    const uint64_t cw = rr < 8 ? codes : codes_hi;
+                    st_entry(&rq[pw][rr][pos & (QN - 1)], ent | (uint32_t)((cw >> (8 * (rr & 7))) & 0xFFu) << 16 |
                                                                (uint32_t)(((pos / QN) & 1) ^ 1) << 31);
                 }
                 tails[rr] += __popc(bal);
@@ -564,7 +565,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 PairEntry nxt;                             // prefetch the next round's entry
                 if (lane < round && q + round < n) nxt = entry(q + round);
                 uint32_t mask = 0, ent = 0;
-                uint64_t codes = 0;                         // in a register (an array was spilled)
+                uint64_t codes = 0, codes_hi = 0;           // in registers (an array was spilled)
                 if (act) {
                     int s = sl + lane, use = wraps;
                     if (s >= nslp) { s -= nslp; use++; }
@@ -587,8 +588,9 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                         mask = cur.mask;
                         M.e.U0 = cur.U0;
                         M.e.U1 = cur.U1;
-                        static_assert(kPairRows <= 8, "codes packing");
+                        static_assert(kPairRows == 8 || kPairRows == 16, "codes packing");
                         codes = *reinterpret_cast<const uint64_t *>(cur.code);
+                        if (kPairRows > 8) codes_hi = *reinterpret_cast<const uint64_t *>(cur.code + 8);
                         // rows that do not read the slot release it now
                         if (__popc(mask) < kPairRows) mbar_arrive_cnt(empty0 + 8 * s, kPairRows - __popc(mask));
                         mbar_arrive_expect_tx(full0 + 8 * s, seg_bytes);
@@ -611,7 +613,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                     }
                 }
                 const long long tpu = prof ? clock64() : 0;
-                push(act, mask, ent, codes);
+                push(act, mask, ent, codes, codes_hi);
                 if (prof && lane == 0) t_push += clock64() - tpu;
                 cur = nxt;
                 const int adv = min(round, stages - r0);
@@ -629,7 +631,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 ent = (uint32_t)sg_ | (uint32_t)(wraps & 1) << 6 | 128u;   // control slot
                 mbar_arrive(full0 + 8 * sg_);
             }
-            push(act, (1u << kPairRows) - 1u, ent, 0ull);
+            push(act, (1u << kPairRows) - 1u, ent, 0ull, 0ull);
         }
         if (prof && lane == 0) {
             atomicAdd(prof + 0, (unsigned long long)(clock64() - t_p0));
