@@ -359,24 +359,27 @@ static_assert(sizeof(PairMeta) == 64, "PairMeta size");
 // chunk j, in the slot (precomputed once); S reads row p, levels m + d: the same
 // offset + NMP*8 + 8d.  S candidates with m + d > n_m - 1 are read (in bounds of
 // the padded ring) and discarded by predicate, so the code has no per-lane branch.
-template <int NMP>
+template <int NMP, bool TWO>
 __device__ __forceinline__ void pair_relax(double (&b0)[NMP], double (&b1)[NMP], const char *slot,
                                            const int (&off0)[NMP / 2], const int (&off1)[NMP / 2],
                                            const int (&m2)[NMP / 2], int d, bool nf, double U, int lim) {
-    // both processor rows of the thread at once: the S validity predicates (which depend
-    // on the lane's chunk rotation, not on the row) are formed once per chunk, and each
-    // is folded into the candidate's compare (one DSETP with a predicate operand and one
-    // 64-bit select per level, rather than a second select for the predicate)
+    // both processor rows of the thread at once (TWO; one row when the tile has <= 32
+    // processor rows): the S validity predicates (which depend on the lane's chunk
+    // rotation, not on the row) are formed once per chunk, and each is folded into the
+    // candidate's compare (one DSETP with a predicate operand and one 64-bit select per
+    // level, rather than a second select for the predicate)
     constexpr int C = NMP / 2;
     if (nf) {                                                    // N
 #pragma unroll
         for (int c = 0; c < C; c++) {
             const double2 x = *reinterpret_cast<const double2 *>(slot + off0[c]);
-            const double2 y = *reinterpret_cast<const double2 *>(slot + off1[c]);
             b0[2 * c] = dmin(b0[2 * c], x.x);
             b0[2 * c + 1] = dmin(b0[2 * c + 1], x.y);
-            b1[2 * c] = dmin(b1[2 * c], y.x);
-            b1[2 * c + 1] = dmin(b1[2 * c + 1], y.y);
+            if (TWO) {
+                const double2 y = *reinterpret_cast<const double2 *>(slot + off1[c]);
+                b1[2 * c] = dmin(b1[2 * c], y.x);
+                b1[2 * c + 1] = dmin(b1[2 * c + 1], y.y);
+            }
         }
     }
     if (lim >= 0) {                                              // S: valid iff m <= lim = n_m-1-d
@@ -384,33 +387,45 @@ __device__ __forceinline__ void pair_relax(double (&b0)[NMP], double (&b1)[NMP],
 #pragma unroll
         for (int c = 0; c < C; c++) {
             const bool v0 = m2[c] <= lim, v1 = m2[c] + 1 <= lim;
-            double y0, y1, z0, z1;
+            double y0, y1, z0 = 0.0, z1 = 0.0;
             if ((d & 1) == 0) {
                 const double2 y = *reinterpret_cast<const double2 *>(srow + off0[c]);
-                const double2 z = *reinterpret_cast<const double2 *>(srow + off1[c]);
-                y0 = y.x; y1 = y.y; z0 = z.x; z1 = z.y;
+                y0 = y.x; y1 = y.y;
+                if (TWO) {
+                    const double2 z = *reinterpret_cast<const double2 *>(srow + off1[c]);
+                    z0 = z.x; z1 = z.y;
+                }
             } else {
                 y0 = *reinterpret_cast<const double *>(srow + off0[c]);
                 y1 = *reinterpret_cast<const double *>(srow + off0[c] + 8);
-                z0 = *reinterpret_cast<const double *>(srow + off1[c]);
-                z1 = *reinterpret_cast<const double *>(srow + off1[c] + 8);
+                if (TWO) {
+                    z0 = *reinterpret_cast<const double *>(srow + off1[c]);
+                    z1 = *reinterpret_cast<const double *>(srow + off1[c] + 8);
+                }
             }
             const double c0 = __dadd_rn(U, y0), c1 = __dadd_rn(U, y1);
-            const double e0 = __dadd_rn(U, z0), e1 = __dadd_rn(U, z1);
             // b = (valid && cand < b) ? cand : b, the validity folded into the compare
             asm("{\n\t.reg .pred q0, q1, p;\n\t"
-                "setp.ne.u32 q0, %8, 0;\n\t"
-                "setp.ne.u32 q1, %9, 0;\n\t"
-                "setp.lt.and.f64 p, %4, %0, q0;\n\t"
-                "selp.f64 %0, %4, %0, p;\n\t"
-                "setp.lt.and.f64 p, %5, %1, q1;\n\t"
-                "selp.f64 %1, %5, %1, p;\n\t"
-                "setp.lt.and.f64 p, %6, %2, q0;\n\t"
-                "selp.f64 %2, %6, %2, p;\n\t"
-                "setp.lt.and.f64 p, %7, %3, q1;\n\t"
-                "selp.f64 %3, %7, %3, p;\n\t}"
-                : "+d"(b0[2 * c]), "+d"(b0[2 * c + 1]), "+d"(b1[2 * c]), "+d"(b1[2 * c + 1])
-                : "d"(c0), "d"(c1), "d"(e0), "d"(e1), "r"((unsigned)v0), "r"((unsigned)v1));
+                "setp.ne.u32 q0, %4, 0;\n\t"
+                "setp.ne.u32 q1, %5, 0;\n\t"
+                "setp.lt.and.f64 p, %2, %0, q0;\n\t"
+                "selp.f64 %0, %2, %0, p;\n\t"
+                "setp.lt.and.f64 p, %3, %1, q1;\n\t"
+                "selp.f64 %1, %3, %1, p;\n\t}"
+                : "+d"(b0[2 * c]), "+d"(b0[2 * c + 1])
+                : "d"(c0), "d"(c1), "r"((unsigned)v0), "r"((unsigned)v1));
+            if (TWO) {
+                const double e0 = __dadd_rn(U, z0), e1 = __dadd_rn(U, z1);
+                asm("{\n\t.reg .pred q0, q1, p;\n\t"
+                    "setp.ne.u32 q0, %4, 0;\n\t"
+                    "setp.ne.u32 q1, %5, 0;\n\t"
+                    "setp.lt.and.f64 p, %2, %0, q0;\n\t"
+                    "selp.f64 %0, %2, %0, p;\n\t"
+                    "setp.lt.and.f64 p, %3, %1, q1;\n\t"
+                    "selp.f64 %1, %3, %1, p;\n\t}"
+                    : "+d"(b1[2 * c]), "+d"(b1[2 * c + 1])
+                    : "d"(e0), "d"(e1), "r"((unsigned)v0), "r"((unsigned)v1));
+            }
         }
     }
 }
@@ -463,7 +478,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     __shared__ __align__(8) uint64_t full[kPairSlotsMax];
     __shared__ __align__(8) uint64_t empty[kPairSlotsMax];
     __shared__ __align__(16) PairMeta meta[kPairSlotsMax];
-    // per-row queues: slot | parity << 6 | control << 7 | n_m << 8 | code << 16 | wrap bit << 31
+    // per-row queues: slot | parity << 6 | control << 7 | n_m << 8 | two rows << 12 | code << 16 | wrap bit << 31
     __shared__ uint32_t rq[kPairProd][kPairRows][QN];
     __shared__ __align__(128) PairEntry stage[kPairProd][2][kPairStage];   // list heads of this and the next tile
     __shared__ __align__(8) uint64_t stbar[kPairProd][2];
@@ -577,8 +592,9 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                         const unsigned mx = __reduce_max_sync(__activemask(), dw);
                         if (lane == 0) t_we += mx;
                     }
-                    // queue entry: slot | parity << 6 | control << 7 | n_m << 8 | row code << 16 (n_m <= 8)
-                    ent = (uint32_t)s | (uint32_t)(use & 1) << 6 | (uint32_t)hd.n_m << 8;
+                    // queue entry: slot | parity << 6 | control << 7 | n_m << 8 (n_m <= 8) | np > 32 << 12 |
+                    // row code << 16
+                    ent = (uint32_t)s | (uint32_t)(use & 1) << 6 | (uint32_t)hd.n_m << 8 | (np > 32 ? 4096u : 0u);
                     PairMeta &M = meta[s];
                     if (q < n) {
                         bulk_g2s(ring_s + 8u * (uint32_t)(s * seg_doubles),
@@ -718,7 +734,10 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             const double U = isB ? M.e.U1 : M.e.U0;
             const int lim = (int)((ent >> 8) & 15u) - 1 - d;   // n_m - 1 - d
             const char *slot = ring + s * seg_bytes;
-            pair_relax<NMP>(b0, b1, slot, off0, off1, m2, d, nf, U, lim);
+            if (ent & 4096u)                               // the tile has > 32 processor rows
+                pair_relax<NMP, true>(b0, b1, slot, off0, off1, m2, d, nf, U, lim);
+            else
+                pair_relax<NMP, false>(b0, b1, slot, off0, off1, m2, d, nf, U, lim);
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(empty0 + 8 * s);

@@ -1,0 +1,29 @@
+#!/usr/bin/env python
+"""Build the compile-time A/B variants of libmadpipe as their own in-tree libraries
+(paper_conf_ipps_beaumontes22_b200/libmadpipe_<name>.so, flags stamped in <lib>.flags),
+for scripts/gpu_variants.sh.  Every variant must pass the pair-path parity tests before
+it is timed; the defaults in the sources are the variants that won.
+
+    python scripts/build_variants.py [name ...]      (default: all)
+"""
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+VARIANTS = {
+    "base": "",                                   # the defaults
+    "vb8": "-DMP_PAIR_VB=8",                      # 8 delay rows x 2 layers per tile, 1 CTA per SM
+    "qatomic": "-DMP_QUEUE_ATOMIC=1",             # queue words through shared atomics (racecheck-clean)
+    "noprof": "-DMP_PAIR_PROF=0",                 # cycle counters compiled out
+    "poll0": "-DMP_POLL_NS=0",                    # consumers spin without back-off
+}
+
+if __name__ == "__main__":
+    names = sys.argv[1:] or list(VARIANTS)
+    for n in names:
+        lib = os.path.join(ROOT, "paper_conf_ipps_beaumontes22_b200", "libmadpipe_%s.so" % n)
+        env = dict(os.environ, MADPIPE_DEFS=VARIANTS[n], MADPIPE_LIB=lib)
+        subprocess.check_call([sys.executable, "-c", "from paper_conf_ipps_beaumontes22_b200 import build; "
+                               "print(build.build(force=True))"], cwd=ROOT, env=env)
+        print(n, VARIANTS[n] or "(defaults)")
