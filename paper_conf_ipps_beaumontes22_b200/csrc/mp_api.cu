@@ -441,6 +441,24 @@ void tile_geom(int P, int n_v, int *vb, int *np, int *n_ptiles, int *n_tiles) {
     *n_tiles = ((n_v + *vb - 1) / *vb) * *n_ptiles;
 }
 
+// Step kernel of a job (measured): the persistent TMA kernel moves one row
+// segment per stage, which pays off from ~1 KB segments; below, plain loads win; the
+// two-layer kernel where it measured faster: P > 33 at GPT shape (profiles/r01_pair_dispatch.md)
+// and, with its one-row-per-thread mode for tiles of <= 32 processors, from P = 17 on the
+// config-5 batch (profiles/r02_batch.md), n_mem <= 8.  MADPIPE_KERNEL forces one (falling
+// back where it does not apply).
+int step_kernel_for(const madpipe_ctx *ctx, int P, int nmp, int n_v, int all_maxL) {
+    int k = ctx->kernel;
+    if (k == 3 && !pair_supported(P, nmp, n_v, all_maxL)) k = -1;
+    if (k < 0) {
+        int vb_, np_, npt_, nt_;
+        persist_geom(P, n_v, nmp, &vb_, &np_, &npt_, &nt_);
+        k = (np_ + 1) * nmp * 8 >= 1024 ? 2 : 0;
+        if (P > 16 && pair_supported(P, nmp, n_v, all_maxL)) k = 3;
+    }
+    return k;
+}
+
 struct BatchHook {
     // called after each batch's tables are complete (before they are reused)
     virtual int after_batch(madpipe_ctx *ctx, const std::vector<int> &job_ids, Job *jobs_dev) {
@@ -477,27 +495,13 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
     const size_t budget = (size_t)ctx->mem_budget;
     // early exit: small first batches that double (time-to-placement); otherwise as
     // many jobs as the table budget holds
-    size_t cap_jobs = early_exit ? (size_t)8 * (size_t)n_chains : SIZE_MAX;
+    size_t cap_jobs = early_exit ? (size_t)std::max(8, 2 * n_chains) : SIZE_MAX;
     int all_maxL = 1;
     for (const auto &c : cs) all_maxL = std::max(all_maxL, (int)c.c.L);
     while (next < js.size()) {
         // ---- form a batch
         hjobs.clear(); htiles.clear(); ids.clear();
-        // step kernel of this batch (measured): the persistent TMA kernel moves
-        // one row segment per stage, which pays off from ~1 KB segments; below, plain loads win;
-        // the two-layer kernel where it measured faster (profiles/r01_pair_dispatch.md): P > 33
-        // (the single-layer kernel needs two warps per delay row there), n_mem <= 8
-        auto kernel_for = [&](int P) {
-            int k = ctx->kernel;
-            if (k == 3 && !pair_supported(P, nmp, disc->n_delay, all_maxL)) k = -1;
-            if (k < 0) {
-                int vb_, np_, npt_, nt_;
-                persist_geom(P, disc->n_delay, nmp, &vb_, &np_, &npt_, &nt_);
-                k = (np_ + 1) * nmp * 8 >= 1024 ? 2 : 0;
-                if (P > 33 && pair_supported(P, nmp, disc->n_delay, all_maxL)) k = 3;
-            }
-            return k;
-        };
+        auto kernel_for = [&](int P) { return step_kernel_for(ctx, P, nmp, disc->n_delay, all_maxL); };
         while (next < js.size() && early_exit && jl_host[js[next].chain] < js[next].j) next++;
         const int kern = next < js.size() ? kernel_for(cs[js[next].chain].P) : 0;
         size_t used = 0;
@@ -1154,9 +1158,18 @@ int batch_sweep(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::v
     for (int j = 0; j < n_c; j++)
         for (int c = 0; c < n; c++)
             if (world == 1 || owner[(size_t)c * n_c + j] == rank) js.push_back({c, j});
-    // group by P (a step launch runs one tile geometry); within a group candidate-major
-    std::stable_sort(js.begin(), js.end(),
-                     [&](const JobSpec &a, const JobSpec &b) { return cs[a.chain].P < cs[b.chain].P; });
+    // group by step kernel (one kernel per launch; the single-layer persistent kernel also
+    // needs one P per launch); within a group candidate-major, so that with early exit the
+    // first batches hold every chain's cheapest candidates
+    const int nmp = nmp_of(disc->n_mem);
+    int all_maxL = 1;
+    for (const auto &c : cs) all_maxL = std::max(all_maxL, (int)c.c.L);
+    std::vector<int> grp(n);
+    for (int c = 0; c < n; c++) {
+        const int k = step_kernel_for(ctx, cs[c].P, nmp, disc->n_delay, all_maxL);
+        grp[c] = k * 65536 + (k == 2 ? cs[c].P : 0);
+    }
+    std::stable_sort(js.begin(), js.end(), [&](const JobSpec &a, const JobSpec &b) { return grp[a.chain] < grp[b.chain]; });
     cu.assign(n, 0);
     if (js.empty()) return MADPIPE_OK;
     std::vector<uint64_t> counts;

@@ -124,6 +124,9 @@ constexpr int kPairHdr = 2;                      // header entries at the head o
 #ifndef MP_PAIR_PROF
 #define MP_PAIR_PROF 1                                     // MADPIPE_PROF=1 cycle counters in pair_step_kernel
 #endif
+#ifndef MP_PAIR_ONEROW
+#define MP_PAIR_ONEROW 1                                   // one processor row per thread for tiles of <= 32
+#endif
 #ifndef MP_PAIR_STAGE
 #define MP_PAIR_STAGE 32
 #endif
@@ -594,7 +597,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                     }
                     // queue entry: slot | parity << 6 | control << 7 | n_m << 8 (n_m <= 8) | np > 32 << 12 |
                     // row code << 16
-                    ent = (uint32_t)s | (uint32_t)(use & 1) << 6 | (uint32_t)hd.n_m << 8 | (np > 32 ? 4096u : 0u);
+                    ent = (uint32_t)s | (uint32_t)(use & 1) << 6 | (uint32_t)hd.n_m << 8 | (np > 32 || !MP_PAIR_ONEROW ? 4096u : 0u);
                     PairMeta &M = meta[s];
                     if (q < n) {
                         bulk_g2s(ring_s + 8u * (uint32_t)(s * seg_doubles),

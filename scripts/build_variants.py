@@ -17,6 +17,7 @@ VARIANTS = {
     "qatomic": "-DMP_QUEUE_ATOMIC=1",             # queue words through shared atomics (racecheck-clean)
     "noprof": "-DMP_PAIR_PROF=0",                 # cycle counters compiled out
     "poll0": "-DMP_POLL_NS=0",                    # consumers spin without back-off
+    "tworow": "-DMP_PAIR_ONEROW=0",               # always relax both processor rows of a thread
 }
 
 if __name__ == "__main__":

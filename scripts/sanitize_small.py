@@ -4,7 +4,7 @@ Covers every kernel the library dispatches:
   * the toy config (step_kernel v1), early_exit=2, a table export;
   * fuzz chains across every NMP template and mode on the default dispatch;
   * the two-layer path (pair_trans / pair_step / pair_fixup): P = 40 and 64 with
-    n_mem <= 8 and L >= 4 -- default dispatch (P > 33), plus small fuzz cases with
+    n_mem <= 8 and L >= 4 -- default dispatch (P > 16), plus small fuzz cases with
     MADPIPE_KERNEL=pair forced, a mixed-length solve_batch (tiles of finished
     chains skipped), early_exit = 2, a tiny ring round (MADPIPE_PAIR_ROUND=1:
     every slot its own round, the producer wraps the ring most often);
@@ -59,7 +59,7 @@ if "base" in parts:
         print("batch", [x["cand_index"] for x in ctx.solve_batch(chains, [4, 6, 9], [10**10, 2 * 10**10, 5 * 10**9],
                                                                   [10e9, 20e9, 50e9], 8, 32, 16)])
 if "pair" in parts:
-    with mp.Context(0) as ctx:                                   # default dispatch: P > 33 -> pair
+    with mp.Context(0) as ctx:                                   # default dispatch: P > 16 -> pair
         for P, n_m, n_v, L in ((40, 8, 48, 12), (64, 8, 64, 10), (40, 4, 33, 7), (70, 5, 20, 9)):
             c2 = chaingen.tiny(rng, L, a_hi=200)
             r = ctx.solve(c2, P, mem_of(c2, 0.5), 25.0, n_m, n_v, 6)
