@@ -63,6 +63,7 @@ struct madpipe_ctx {
     int prof = 0;             // MADPIPE_PROF=1: cycle counters of the persistent step kernel to stderr
     int n_prod = 4;           // MADPIPE_NPROD: producer warps of the persistent step kernel (1..4)
     int tile_block = 1;       // MADPIPE_TILE_BLOCK: consecutive tiles per interleaved block (1 = round-robin)
+    int trans_overlap = 1;    // MADPIPE_TRANS_OVERLAP: pair path builds pass i+1's lists beside step(i) (1) or after it (0)
     DevBuf profbuf;
     int num_sms = 148;
     int n_rec = 0;            // step-kernel launches bracketed by per-launch events in the last batch
@@ -273,6 +274,7 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, int32_t rank, i
     c->prof = pf && pf[0] == '1';
     if (const char *e = getenv("MADPIPE_NPROD")) c->n_prod = std::max(1, std::min(4, atoi(e)));
     if (const char *e = getenv("MADPIPE_TILE_BLOCK")) c->tile_block = std::max(1, atoi(e));
+    if (const char *e = getenv("MADPIPE_TRANS_OVERLAP")) c->trans_overlap = atoi(e) != 0;
     cudaEventCreate(&c->ev_a);
     cudaEventCreate(&c->ev_b);
     cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking);
@@ -691,18 +693,29 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             ctx->launches++;
             int n_rec = 0;
             const int cap = pair_list_cap(maxL);
-            // pass i covers layers l = 2i+1, l+1 with list buffer i % 2:
-            //   stream: [wait trans(i)] step(i) -> fixup(i)
-            //   aux:    [wait step(i)]  trans(i+1)
-            // trans(i+1) writes list buffer (i+1) % 2 (last read by step(i-1)), reads the
-            // final flags of slabs <= l and, for slab l+1, a superset of what fixup(i)
-            // will flag (pair_trans_kernel, fix_slab).  (Measured: the two kernels hardly
-            // overlap, and one launch with their blocks interleaved was slower, 6.3.)
-            launch_pair_trans(djobs, nj, n_v_max, 1, nmp, 0, -1, ctx->stream);
+            // pass i covers layers l = 2i+1, l+1 with list buffer i % 2.
+            // trans_overlap = 1 (default):
+            //   stream: [wait trans(i)] (mark) step(i) -> fixup(i)
+            //   aux:    [wait mark]     trans(i+1)     -- runs beside step(i)
+            //   trans(i+1) needs the final slabs <= l-1 (fixup(i-1) precedes the mark) and keeps
+            //   every live entry reading slabs l, l+1 unverified (unv_from = l); it writes list
+            //   buffer (i+1) % 2, last read by step(i-1).
+            // trans_overlap = 0 (round 1):
+            //   aux:    [wait step(i)]  trans(i+1)     -- beside fixup(i); it reads the final flags of
+            //   slabs <= l and, for slab l+1, a superset of what fixup(i) will flag (fix_slab).
+            launch_pair_trans(djobs, nj, n_v_max, 1, nmp, 0, -1, INT_MAX, ctx->stream);
             ctx->launches++;
             for (int l = 1; l <= maxL; l += 2) {
                 const int i = l >> 1, b = i & 1;
                 if (i >= 1) CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->stream, ctx->ev_tr[b], 0));
+                if (ctx->trans_overlap && l + 2 <= maxL) {
+                    CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[b], ctx->stream));
+                    CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_st[b], 0));
+                    launch_pair_trans(djobs, nj, n_v_max, l + 2, nmp, (size_t)(b ^ 1) * list_buf_entries, -1, l,
+                                      ctx->aux);
+                    CUDA_TRY(ctx, cudaEventRecord(ctx->ev_tr[b ^ 1], ctx->aux));
+                    ctx->launches++;
+                }
                 if (per_launch) cudaEventRecord(ctx->ev_pool[2 * n_rec], ctx->stream);
                 launch_pair_step((const int2 *)ctx->tdesc.p, n_tiles, ctx->tlist.p, b * list_buf_entries, cap, nmp,
                                  p_np, nsg, persist_grid,
@@ -711,11 +724,11 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                 if (per_launch) cudaEventRecord(ctx->ev_pool[2 * n_rec + 1], ctx->stream);
                 n_rec++;
                 ctx->launches++;
-                if (l + 2 <= maxL) {
+                if (!ctx->trans_overlap && l + 2 <= maxL) {
                     CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[b], ctx->stream));
                     CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_st[b], 0));
                     launch_pair_trans(djobs, nj, n_v_max, l + 2, nmp, (size_t)(b ^ 1) * list_buf_entries, l + 1,
-                                      ctx->aux);
+                                      INT_MAX, ctx->aux);
                     CUDA_TRY(ctx, cudaEventRecord(ctx->ev_tr[b ^ 1], ctx->aux));
                     ctx->launches++;
                 }
@@ -891,6 +904,17 @@ int resolve_impl(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::
     for (int c = 0; c < (int)cs.size(); c++) {
         maxL = std::max(maxL, (int)cs[c].c.L);
         if (jstar[c] != INT32_MAX && jstar[c] >= 0) js.push_back({c, jstar[c]});
+    }
+    // group the winners by step kernel (and P on the single-layer persistent kernel), as
+    // batch_sweep does, so that they run as a few batches and not one per kernel change
+    {
+        const int nmp = nmp_of(disc->n_mem);
+        std::stable_sort(js.begin(), js.end(), [&](const JobSpec &a, const JobSpec &b) {
+            const int ka = step_kernel_for(ctx, cs[a.chain].P, nmp, disc->n_delay, maxL);
+            const int kb = step_kernel_for(ctx, cs[b.chain].P, nmp, disc->n_delay, maxL);
+            const int ga = ka * 65536 + (ka == 2 ? cs[a.chain].P : 0), gb = kb * 65536 + (kb == 2 ? cs[b.chain].P : 0);
+            return ga < gb;
+        });
     }
     TraceHook hook;
     hook.nmp = nmp_of(disc->n_mem);

@@ -176,7 +176,11 @@ __device__ __forceinline__ int pair_vtiles(int n_v) { return (n_v + kPairVB - 1)
 // a3 + a4 for the layer pair (l, l+1).
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, int l, int nmp, size_t buf_off,
-                                                int fix_slab) {
+                                                int fix_slab, int unv_from) {
+    // unv_from: source slabs >= unv_from are still being written by the step (and fixup)
+    // kernels of the previous pass when this launch overlaps them (MADPIPE_TRANS_OVERLAP):
+    // their row flags are not consulted and every live entry reading them is kept (a
+    // superset of the useful ones, so the skip stays exact).
     // fix_slab (= l-1, or -1): this launch runs concurrently with pair_fixup_kernel of
     // slab fix_slab, which may still turn that slab's row flags on.  For a source row w
     // of that slab whose flag is still 0, the entry is kept if the fixup could make the
@@ -266,6 +270,7 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
 #pragma unroll
         for (int u = 0; u < TU; u++) {
             const int sk = (key[u] >> 16) - 1;   // source slab
+            if (key[u] >= 0 && sk >= unv_from) fl[u] = 1u;
             if (key[u] >= 0 && fl[u] == 0u && sk == fix_slab && sk >= J.kwin[sk]) {
                 const int w = key[u] & 0xFFFF;
                 int64_t d2;
@@ -329,13 +334,13 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
 #define MP_TRANS_MINB 8
 #endif
 __global__ void __launch_bounds__(128, MP_TRANS_MINB) pair_trans_kernel(const Job *jobs, int l, int nmp, size_t buf_off,
-                                                         int fix_slab) {
+                                                         int fix_slab, int unv_from) {
     __shared__ Job sJ;
     if (threadIdx.x < sizeof(Job) / 8)
         reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
             __ldg(reinterpret_cast<const uint64_t *>(jobs + blockIdx.y) + threadIdx.x);
     __syncthreads();
-    pair_trans_body(sJ, blockIdx.x * 4 + (threadIdx.x >> 5), threadIdx.x & 31, l, nmp, buf_off, fix_slab);
+    pair_trans_body(sJ, blockIdx.x * 4 + (threadIdx.x >> 5), threadIdx.x & 31, l, nmp, buf_off, fix_slab, unv_from);
 }
 
 // ---------------------------------------------------------------------------
@@ -849,9 +854,9 @@ bool pair_supported(int P, int nmp, int n_v, int max_L) {
 }
 
 void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int fix_slab,
-                       cudaStream_t s) {
+                       int unv_from, cudaStream_t s) {
     const int nvt = (n_v_max + kPairVB - 1) / kPairVB + kPairE;
-    pair_trans_kernel<<<dim3((nvt + 3) / 4, n_jobs), 128, 0, s>>>(jobs, l, nmp, buf_off, fix_slab);
+    pair_trans_kernel<<<dim3((nvt + 3) / 4, n_jobs), 128, 0, s>>>(jobs, l, nmp, buf_off, fix_slab, unv_from);
 }
 
 void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, cudaStream_t s) {
