@@ -178,6 +178,13 @@ def oracle_baseline(cfg, one_core=True):
     out["full_sweep_cell_updates"] = total
     off = _offline_seconds(cfg)
     if off is not None:
+        sam = json.load(open(os.path.join(ROOT, "configs", "gpt_oracle_samples.json")))["samples"]
+        out["stratified_sample_offline"] = {
+            "candidates": [r["j"] for r in sam], "cell_updates": sum(r["cell_updates"] for r in sam),
+            "oracle_1thread_s": sum(r["oracle_s"] for r in sam),
+            "rate_1thread": sum(r["cell_updates"] for r in sam) / sum(r["oracle_s"] for r in sam),
+            "what": "SURVEY 8(d) GPT sample (j <= j*, j*+1..8, 16 stratified above, 511/767/1023), each "
+                    "candidate's full table by the oracle on 1 thread (8 at a time), scripts/oracle_gpt_samples.py"}
         # the oracle's rate grows with j (longer windows, more skipped transitions), so the
         # full sweep is extrapolated from the stratified per-candidate times measured
         # offline, rescaled to this host by the live 1-core scan of j = 0..j*

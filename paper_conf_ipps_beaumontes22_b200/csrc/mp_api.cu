@@ -63,7 +63,8 @@ struct madpipe_ctx {
     int prof = 0;             // MADPIPE_PROF=1: cycle counters of the persistent step kernel to stderr
     int n_prod = 4;           // MADPIPE_NPROD: producer warps of the persistent step kernel (1..4)
     int tile_block = 1;       // MADPIPE_TILE_BLOCK: consecutive tiles per interleaved block (1 = round-robin)
-    int trans_overlap = 1;    // MADPIPE_TRANS_OVERLAP: pair path builds pass i+1's lists beside step(i) (1) or after it (0)
+    int trans_overlap = 0;    // MADPIPE_TRANS_OVERLAP=1: pair path builds pass i+1's lists beside step(i) (measured
+                              // slower at GPT: 909 vs 886 ms, 5% more entries kept unverified + contention)
     DevBuf profbuf;
     int num_sms = 148;
     int n_rec = 0;            // step-kernel launches bracketed by per-launch events in the last batch
@@ -434,12 +435,14 @@ size_t table_doubles(const ChainSpec &c, const madpipe_disc *disc) {
     return (size_t)(c.c.L + 1) * (size_t)disc->n_delay * (size_t)c.P * (size_t)nmp_of(disc->n_mem);
 }
 
-// Tile geometry of one job: np processor rows x vb delay rows.
-void tile_geom(int P, int n_v, int *vb, int *np, int *n_ptiles, int *n_tiles) {
+// Tile geometry of one job on the plain-load kernel: np processor rows x vb delay rows,
+// one thread each, for CTAs of `threads` threads (128 when every chain of the batch has
+// P <= 16, so that small tiles do not leave most of a 256-thread CTA idle).
+void tile_geom(int P, int n_v, int threads, int *vb, int *np, int *n_ptiles, int *n_tiles) {
     const int rows = std::max(1, P - 1);
-    *np = std::min(rows, kThreads);
+    *np = std::min(rows, threads);
     *n_ptiles = (rows + *np - 1) / *np;
-    *vb = std::max(1, std::min(n_v, kThreads / *np));
+    *vb = std::max(1, std::min(n_v, threads / *np));
     *n_tiles = ((n_v + *vb - 1) / *vb) * *n_ptiles;
 }
 
@@ -504,6 +507,10 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
         // ---- form a batch
         hjobs.clear(); htiles.clear(); ids.clear();
         auto kernel_for = [&](int P) { return step_kernel_for(ctx, P, nmp, disc->n_delay, all_maxL); };
+        // CTA size of the plain-load kernel: 128 threads if every chain on it has P <= 17
+        int v1_threads = 128;
+        for (const auto &c : cs)
+            if (c.P > 17 && kernel_for(c.P) == 0) v1_threads = kThreads;
         while (next < js.size() && early_exit && jl_host[js[next].chain] < js[next].j) next++;
         const int kern = next < js.size() ? kernel_for(cs[js[next].chain].P) : 0;
         size_t used = 0;
@@ -538,7 +545,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             } else if (kern == 2) {
                 persist_geom(c.P, disc->n_delay, nmp, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
             } else {
-                tile_geom(c.P, disc->n_delay, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
+                tile_geom(c.P, disc->n_delay, v1_threads, &J.vb, &J.np, &J.n_ptiles, &n_tiles);
             }
             J.tile0 = (int32_t)htiles.size();
             for (int t = 0; t < n_tiles; t++) htiles.push_back((int32_t)hjobs.size());
@@ -694,13 +701,13 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             int n_rec = 0;
             const int cap = pair_list_cap(maxL);
             // pass i covers layers l = 2i+1, l+1 with list buffer i % 2.
-            // trans_overlap = 1 (default):
+            // trans_overlap = 1 (MADPIPE_TRANS_OVERLAP=1; measured slower):
             //   stream: [wait trans(i)] (mark) step(i) -> fixup(i)
             //   aux:    [wait mark]     trans(i+1)     -- runs beside step(i)
             //   trans(i+1) needs the final slabs <= l-1 (fixup(i-1) precedes the mark) and keeps
             //   every live entry reading slabs l, l+1 unverified (unv_from = l); it writes list
             //   buffer (i+1) % 2, last read by step(i-1).
-            // trans_overlap = 0 (round 1):
+            // trans_overlap = 0 (default, round 1):
             //   aux:    [wait step(i)]  trans(i+1)     -- beside fixup(i); it reads the final flags of
             //   slabs <= l and, for slab l+1, a superset of what fixup(i) will flag (fix_slab).
             launch_pair_trans(djobs, nj, n_v_max, 1, nmp, 0, -1, INT_MAX, ctx->stream);
@@ -763,7 +770,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                                     persist_grid, (unsigned long long *)(ctx->prof ? ctx->profbuf.p : nullptr),
                                     ctx->n_prod, ctx->tile_block, buf_off, ctx->stream);
             else
-                launch_step(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, ctx->stream);
+                launch_step(djobs, (const int32_t *)ctx->tiles.p, n_tiles, l, nmp, v1_threads, ctx->stream);
             if (per_launch) cudaEventRecord(ctx->ev_pool[2 * (l - 1) + 1], ctx->stream);
             if (kern == 2) CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[l & 3], ctx->stream));
         }

@@ -86,7 +86,7 @@ __host__ __device__ inline int32_t pack_trans(int vn, int64_t d, bool nf) {
 void launch_prep(ChainDev *chains_dev, int n_chains, cudaStream_t s);
 void launch_jobs_init(Job *jobs, int n_jobs, cudaStream_t s);
 void launch_init_slab0(const Job *jobs, int n_jobs, int nmp, int max_cells, cudaStream_t s);
-void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp,
+void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int threads,
                  cudaStream_t s);
 void launch_step_persist(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int np,
                          int vb, int nsg, int grid, unsigned long long *prof, int n_prod, int tile_block,

@@ -185,7 +185,7 @@ __global__ void __launch_bounds__(kThreads) step_kernel(const Job *__restrict__ 
         const int nk = min(kc_len, l + 1 - kc0);
         __syncthreads();
         unsigned live = 0;
-        for (int e = tid; e < nk * vcount; e += kThreads) {
+        for (int e = tid; e < nk * vcount; e += blockDim.x) {
             const int kk = e / vcount, v2 = e - kk * vcount;
             const int k = kc0 + kk;
             const double Ukl = __dsub_rn(Ul, J.Up[k - 1]);
@@ -242,15 +242,15 @@ __global__ void __launch_bounds__(kThreads) step_kernel(const Job *__restrict__ 
     }
 }
 
-void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp,
+void launch_step(const Job *jobs, const int32_t *tile_job, int n_tiles, int l, int nmp, int threads,
                  cudaStream_t s) {
     switch (nmp) {
-    case 2: step_kernel<2><<<n_tiles, kThreads, 0, s>>>(jobs, tile_job, l); break;
-    case 4: step_kernel<4><<<n_tiles, kThreads, 0, s>>>(jobs, tile_job, l); break;
-    case 8: step_kernel<8><<<n_tiles, kThreads, 0, s>>>(jobs, tile_job, l); break;
-    case 16: step_kernel<16><<<n_tiles, kThreads, 0, s>>>(jobs, tile_job, l); break;
-    case 32: step_kernel<32><<<n_tiles, kThreads, 0, s>>>(jobs, tile_job, l); break;
-    default: step_kernel<64><<<n_tiles, kThreads, 0, s>>>(jobs, tile_job, l); break;
+    case 2: step_kernel<2><<<n_tiles, threads, 0, s>>>(jobs, tile_job, l); break;
+    case 4: step_kernel<4><<<n_tiles, threads, 0, s>>>(jobs, tile_job, l); break;
+    case 8: step_kernel<8><<<n_tiles, threads, 0, s>>>(jobs, tile_job, l); break;
+    case 16: step_kernel<16><<<n_tiles, threads, 0, s>>>(jobs, tile_job, l); break;
+    case 32: step_kernel<32><<<n_tiles, threads, 0, s>>>(jobs, tile_job, l); break;
+    default: step_kernel<64><<<n_tiles, threads, 0, s>>>(jobs, tile_job, l); break;
     }
 }
 
