@@ -124,6 +124,9 @@ constexpr int kPairHdr = 2;                      // header entries at the head o
 #ifndef MP_PAIR_PROF
 #define MP_PAIR_PROF 1                                     // MADPIPE_PROF=1 cycle counters in pair_step_kernel
 #endif
+#ifndef MP_PAIR_L2PF
+#define MP_PAIR_L2PF 3                                     // list entries prefetched into L2, in producer rounds
+#endif
 #ifndef MP_PAIR_ONEROW
 #define MP_PAIR_ONEROW 1                                   // one processor row per thread for tiles of <= 32
 #endif
@@ -367,6 +370,58 @@ static_assert(sizeof(PairMeta) == 64, "PairMeta size");
 // chunk j, in the slot (precomputed once); S reads row p, levels m + d: the same
 // offset + NMP*8 + 8d.  S candidates with m + d > n_m - 1 are read (in bounds of
 // the padded ring) and discarded by predicate, so the code has no per-lane branch.
+// S candidates of one slot: b = (valid && U + src[m+d] < b) ? U + src[m+d] : b, the
+// validity folded into the compare (one DSETP with a predicate operand and one 64-bit
+// select per level).  ODD: d is odd, so the shifted levels are not 16-byte aligned.
+template <int NMP, bool TWO, bool ODD>
+__device__ __forceinline__ void pair_relax_s(double (&b0)[NMP], double (&b1)[NMP], const char *srow,
+                                             const int (&off0)[NMP / 2], const int (&off1)[NMP / 2],
+                                             const int (&m2)[NMP / 2], double U, int lim) {
+    constexpr int C = NMP / 2;
+#pragma unroll
+    for (int c = 0; c < C; c++) {
+        const bool v0 = m2[c] <= lim, v1 = m2[c] + 1 <= lim;
+        double y0, y1, z0 = 0.0, z1 = 0.0;
+        if (!ODD) {
+            const double2 y = *reinterpret_cast<const double2 *>(srow + off0[c]);
+            y0 = y.x; y1 = y.y;
+            if (TWO) {
+                const double2 z = *reinterpret_cast<const double2 *>(srow + off1[c]);
+                z0 = z.x; z1 = z.y;
+            }
+        } else {
+            y0 = *reinterpret_cast<const double *>(srow + off0[c]);
+            y1 = *reinterpret_cast<const double *>(srow + off0[c] + 8);
+            if (TWO) {
+                z0 = *reinterpret_cast<const double *>(srow + off1[c]);
+                z1 = *reinterpret_cast<const double *>(srow + off1[c] + 8);
+            }
+        }
+        const double c0 = __dadd_rn(U, y0), c1 = __dadd_rn(U, y1);
+        asm("{\n\t.reg .pred q0, q1, p;\n\t"
+            "setp.ne.u32 q0, %4, 0;\n\t"
+            "setp.ne.u32 q1, %5, 0;\n\t"
+            "setp.lt.and.f64 p, %2, %0, q0;\n\t"
+            "selp.f64 %0, %2, %0, p;\n\t"
+            "setp.lt.and.f64 p, %3, %1, q1;\n\t"
+            "selp.f64 %1, %3, %1, p;\n\t}"
+            : "+d"(b0[2 * c]), "+d"(b0[2 * c + 1])
+            : "d"(c0), "d"(c1), "r"((unsigned)v0), "r"((unsigned)v1));
+        if (TWO) {
+            const double e0 = __dadd_rn(U, z0), e1 = __dadd_rn(U, z1);
+            asm("{\n\t.reg .pred q0, q1, p;\n\t"
+                "setp.ne.u32 q0, %4, 0;\n\t"
+                "setp.ne.u32 q1, %5, 0;\n\t"
+                "setp.lt.and.f64 p, %2, %0, q0;\n\t"
+                "selp.f64 %0, %2, %0, p;\n\t"
+                "setp.lt.and.f64 p, %3, %1, q1;\n\t"
+                "selp.f64 %1, %3, %1, p;\n\t}"
+                : "+d"(b1[2 * c]), "+d"(b1[2 * c + 1])
+                : "d"(e0), "d"(e1), "r"((unsigned)v0), "r"((unsigned)v1));
+        }
+    }
+}
+
 template <int NMP, bool TWO>
 __device__ __forceinline__ void pair_relax(double (&b0)[NMP], double (&b1)[NMP], const char *slot,
                                            const int (&off0)[NMP / 2], const int (&off1)[NMP / 2],
@@ -391,50 +446,11 @@ __device__ __forceinline__ void pair_relax(double (&b0)[NMP], double (&b1)[NMP],
         }
     }
     if (lim >= 0) {                                              // S: valid iff m <= lim = n_m-1-d
+        // the level shift d is the same for the whole warp: one branch on its parity, so each
+        // path issues only its own loads (16-byte pairs for even d, 8-byte singles for odd d)
         const char *srow = slot + NMP * 8 + 8 * d;
-#pragma unroll
-        for (int c = 0; c < C; c++) {
-            const bool v0 = m2[c] <= lim, v1 = m2[c] + 1 <= lim;
-            double y0, y1, z0 = 0.0, z1 = 0.0;
-            if ((d & 1) == 0) {
-                const double2 y = *reinterpret_cast<const double2 *>(srow + off0[c]);
-                y0 = y.x; y1 = y.y;
-                if (TWO) {
-                    const double2 z = *reinterpret_cast<const double2 *>(srow + off1[c]);
-                    z0 = z.x; z1 = z.y;
-                }
-            } else {
-                y0 = *reinterpret_cast<const double *>(srow + off0[c]);
-                y1 = *reinterpret_cast<const double *>(srow + off0[c] + 8);
-                if (TWO) {
-                    z0 = *reinterpret_cast<const double *>(srow + off1[c]);
-                    z1 = *reinterpret_cast<const double *>(srow + off1[c] + 8);
-                }
-            }
-            const double c0 = __dadd_rn(U, y0), c1 = __dadd_rn(U, y1);
-            // b = (valid && cand < b) ? cand : b, the validity folded into the compare
-            asm("{\n\t.reg .pred q0, q1, p;\n\t"
-                "setp.ne.u32 q0, %4, 0;\n\t"
-                "setp.ne.u32 q1, %5, 0;\n\t"
-                "setp.lt.and.f64 p, %2, %0, q0;\n\t"
-                "selp.f64 %0, %2, %0, p;\n\t"
-                "setp.lt.and.f64 p, %3, %1, q1;\n\t"
-                "selp.f64 %1, %3, %1, p;\n\t}"
-                : "+d"(b0[2 * c]), "+d"(b0[2 * c + 1])
-                : "d"(c0), "d"(c1), "r"((unsigned)v0), "r"((unsigned)v1));
-            if (TWO) {
-                const double e0 = __dadd_rn(U, z0), e1 = __dadd_rn(U, z1);
-                asm("{\n\t.reg .pred q0, q1, p;\n\t"
-                    "setp.ne.u32 q0, %4, 0;\n\t"
-                    "setp.ne.u32 q1, %5, 0;\n\t"
-                    "setp.lt.and.f64 p, %2, %0, q0;\n\t"
-                    "selp.f64 %0, %2, %0, p;\n\t"
-                    "setp.lt.and.f64 p, %3, %1, q1;\n\t"
-                    "selp.f64 %1, %3, %1, p;\n\t}"
-                    : "+d"(b1[2 * c]), "+d"(b1[2 * c + 1])
-                    : "d"(e0), "d"(e1), "r"((unsigned)v0), "r"((unsigned)v1));
-            }
-        }
+        if (d & 1) pair_relax_s<NMP, TWO, true>(b0, b1, srow, off0, off1, m2, U, lim);
+        else pair_relax_s<NMP, TWO, false>(b0, b1, srow, off0, off1, m2, U, lim);
     }
 }
 
@@ -587,6 +603,15 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 const bool act = lane < round && q < stages;
                 PairEntry nxt;                             // prefetch the next round's entry
                 if (lane < round && q + round < n) nxt = entry(q + round);
+#if MP_PAIR_L2PF
+                // and pull entries MP_PAIR_L2PF rounds ahead into L2 (lists beyond the staged head
+                // are read from global memory; a DRAM miss there stalls the whole pipeline)
+                {
+                    const int qf = q + MP_PAIR_L2PF * round;
+                    if (lane < round && qf < n && qf + kPairHdr >= stage_n)
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(tl + kPairHdr + qf));
+                }
+#endif
                 uint32_t mask = 0, ent = 0;
                 uint64_t codes = 0, codes_hi = 0;           // in registers (an array was spilled)
                 if (act) {

@@ -18,6 +18,8 @@ VARIANTS = {
     "noprof": "-DMP_PAIR_PROF=0",                 # cycle counters compiled out
     "poll0": "-DMP_POLL_NS=0",                    # consumers spin without back-off
     "tworow": "-DMP_PAIR_ONEROW=0",               # always relax both processor rows of a thread
+    "nol2pf": "-DMP_PAIR_L2PF=0",                 # no L2 prefetch of list entries ahead of the producer
+    "l2pf6": "-DMP_PAIR_L2PF=6",                  # L2 prefetch 6 rounds ahead
 }
 
 if __name__ == "__main__":
