@@ -308,8 +308,9 @@ def main():
     use_dist = world > 1 or args.force_dist
     stream = torch.cuda.current_stream(dev)
     if use_dist:
-        if os.environ.get("NCCL_DEBUG", "VERSION").upper() == "VERSION":
-            os.environ["NCCL_DEBUG"] = "WARN"      # keep stdout to the one JSON line
+        if os.environ.get("NCCL_DEBUG", "VERSION").upper() in ("VERSION", "WARN"):
+            os.environ["NCCL_DEBUG"] = "NONE"      # keep stdout to the one JSON line (VERSION and WARN
+            #                                        both print "NCCL version ..." to stdout at init)
         dist.init_process_group("nccl", device_id=dev)
         ctx = distributed.context(local, stream=stream.cuda_stream)   # ctx-owned NCCL communicator
     else:

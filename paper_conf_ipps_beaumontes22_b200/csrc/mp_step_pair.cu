@@ -83,11 +83,11 @@ __device__ __forceinline__ void mbar_arrive_cnt(uint32_t bar, uint32_t cnt) {
 #ifndef MP_QUEUE_ATOMIC
 #define MP_QUEUE_ATOMIC 0
 #endif
-__device__ __forceinline__ void st_entry(uint32_t *p, uint32_t v) {
+__device__ __forceinline__ void st_entry_s(uint32_t saddr, uint32_t v) {   // shared-window address
 #if MP_QUEUE_ATOMIC
-    asm volatile("atom.shared::cta.exch.b32 _, [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+    asm volatile("atom.shared::cta.exch.b32 _, [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
 #else
-    asm volatile("st.volatile.shared::cta.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+    asm volatile("st.volatile.shared::cta.u32 [%0], %1;" ::"r"(saddr), "r"(v));
 #endif
 }
 __device__ __forceinline__ uint32_t ld_entry(const uint32_t *p) {
@@ -535,21 +535,26 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
 #pragma unroll
         for (int rr = 0; rr < kPairRows; rr++) tails[rr] = 0;
         const unsigned lt = (1u << lane) - 1u;
+        const uint32_t rq_s = smem_u32(&rq[pw][0][0]);     // shared address of this producer's queues
         auto push = [&](bool act, uint32_t mask, uint32_t ent, uint64_t codes, uint64_t codes_hi) {   // byte rr = row rr
             // append ent (+ the row's code, + the wrap bit of its position) to the queue of
-            // every row in mask, in lane order
+            // every row in mask, in lane order.  All ballots first, then the positions and
+            // words, then the stores: independent work the scheduler can overlap.
+            unsigned bal[kPairRows];
+#pragma unroll
+            for (int rr = 0; rr < kPairRows; rr++) bal[rr] = __ballot_sync(0xffffffffu, act && ((mask >> rr) & 1u));
+            uint32_t addr[kPairRows], word[kPairRows];
 #pragma unroll
             for (int rr = 0; rr < kPairRows; rr++) {
-                const bool mine = act && ((mask >> rr) & 1u);
-                const unsigned bal = __ballot_sync(0xffffffffu, mine);
-                if (mine) {
-                    const int pos = tails[rr] + __popc(bal & lt);
-                    const uint64_t cw = rr < 8 ? codes : codes_hi;
-                    st_entry(&rq[pw][rr][pos & (QN - 1)], ent | (uint32_t)((cw >> (8 * (rr & 7))) & 0xFFu) << 16 |
-                                                               (uint32_t)(((pos / QN) & 1) ^ 1) << 31);
-                }
-                tails[rr] += __popc(bal);
+                const int pos = tails[rr] + __popc(bal[rr] & lt);
+                const uint64_t cw = rr < 8 ? codes : codes_hi;
+                addr[rr] = rq_s + 4u * (uint32_t)(rr * QN + (pos & (QN - 1)));
+                word[rr] = ent | (uint32_t)((cw >> (8 * (rr & 7))) & 0xFFu) << 16 | (uint32_t)(((pos / QN) & 1) ^ 1) << 31;
+                tails[rr] += __popc(bal[rr]);
             }
+#pragma unroll
+            for (int rr = 0; rr < kPairRows; rr++)
+                if ((bal[rr] >> lane) & 1u) st_entry_s(addr[rr], word[rr]);
         };
         // prof (MADPIPE_PROF=1): [0] producer cycles, [1] empty-barrier waits (max over lanes),
         // [2] tile setup (header), [3] consumer cycles, [4] queue waits, [5] full waits, [6] data

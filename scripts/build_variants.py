@@ -20,6 +20,8 @@ VARIANTS = {
     "tworow": "-DMP_PAIR_ONEROW=0",               # always relax both processor rows of a thread
     "nol2pf": "-DMP_PAIR_L2PF=0",                 # no L2 prefetch of list entries ahead of the producer
     "l2pf6": "-DMP_PAIR_L2PF=6",                  # L2 prefetch 6 rounds ahead
+    "l2pf2": "-DMP_PAIR_L2PF=2",
+    "l2pf4": "-DMP_PAIR_L2PF=4",
 }
 
 if __name__ == "__main__":
