@@ -108,7 +108,10 @@ __device__ __forceinline__ uint32_t ld_entry(const uint32_t *p) {
 constexpr int kPairVB = MP_PAIR_VB;              // delay rows per layer in a tile
 constexpr int kPairRows = 2 * kPairVB;           // output rows (= consumer warps) per tile
 constexpr int kPairE = 16 / kPairVB;             // extra v-tiles: layer l+1 rows are shifted by <= 16 levels
-constexpr int kPairCtas = 8 / kPairVB;           // resident CTAs per SM (one producer warp each)
+#ifndef MP_PAIR_CTAS
+#define MP_PAIR_CTAS (8 / MP_PAIR_VB)
+#endif
+constexpr int kPairCtas = MP_PAIR_CTAS;           // resident CTAs per SM (one producer warp each)
 constexpr int kPairNp = 64;                      // processor rows per tile (2 per consumer thread)
 constexpr int kPairSlotsMax = kPairVB > 4 ? 48 : 32;  // ring slots (6-bit slot index in the queue word)
 #ifndef MP_PAIR_NPROD
@@ -873,7 +876,7 @@ size_t pair_entry_bytes() { return sizeof(PairEntry); }
 // ring slots per CTA (2 CTAs per SM): as many as fit in ~100 KB
 int pair_nsl(int np, int nmp) {
     const int seg = (np + 1) * nmp * 8;
-    int slots = (200 * 1024 / kPairCtas) / seg;
+    int slots = ((kPairCtas > 2 ? 204 : 200) * 1024 / kPairCtas) / seg;
     slots = slots > kPairSlotsMax ? kPairSlotsMax : slots;
     return slots - slots % kPairProd;                       // split evenly between the producers
 }

@@ -22,6 +22,7 @@ VARIANTS = {
     "l2pf6": "-DMP_PAIR_L2PF=6",                  # L2 prefetch 6 rounds ahead
     "l2pf2": "-DMP_PAIR_L2PF=2",
     "l2pf4": "-DMP_PAIR_L2PF=4",
+    "ctas3": "-DMP_PAIR_CTAS=3",                  # 3 CTAs per SM (16-slot rings, <= 75 registers)
 }
 
 if __name__ == "__main__":
