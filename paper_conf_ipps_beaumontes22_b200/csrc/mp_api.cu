@@ -63,6 +63,9 @@ struct madpipe_ctx {
     int prof = 0;             // MADPIPE_PROF=1: cycle counters of the persistent step kernel to stderr
     int n_prod = 4;           // MADPIPE_NPROD: producer warps of the persistent step kernel (1..4)
     int tile_block = 1;       // MADPIPE_TILE_BLOCK: consecutive tiles per interleaved block (1 = round-robin)
+    // MADPIPE_AUX_GRID=t,f: persistent grids of t and f blocks per SM for the pair path's list
+    // builder and fixup kernels (they run side by side on two streams; 0 = one block per item)
+    int aux_grid_trans = 0, aux_grid_fix = 0;
     int trans_overlap = 0;    // MADPIPE_TRANS_OVERLAP=1: pair path builds pass i+1's lists beside step(i) (measured
                               // slower at GPT: 909 vs 886 ms, 5% more entries kept unverified + contention)
     DevBuf profbuf;
@@ -276,6 +279,10 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, int32_t rank, i
     if (const char *e = getenv("MADPIPE_NPROD")) c->n_prod = std::max(1, std::min(4, atoi(e)));
     if (const char *e = getenv("MADPIPE_TILE_BLOCK")) c->tile_block = std::max(1, atoi(e));
     if (const char *e = getenv("MADPIPE_TRANS_OVERLAP")) c->trans_overlap = atoi(e) != 0;
+    if (const char *e = getenv("MADPIPE_AUX_GRID")) {
+        int t = 0, f = 0;
+        if (sscanf(e, "%d,%d", &t, &f) == 2) { c->aux_grid_trans = t * c->num_sms; c->aux_grid_fix = f * c->num_sms; }
+    }
     cudaEventCreate(&c->ev_a);
     cudaEventCreate(&c->ev_b);
     cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking);
@@ -710,7 +717,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             // trans_overlap = 0 (default, round 1):
             //   aux:    [wait step(i)]  trans(i+1)     -- beside fixup(i); it reads the final flags of
             //   slabs <= l and, for slab l+1, a superset of what fixup(i) will flag (fix_slab).
-            launch_pair_trans(djobs, nj, n_v_max, 1, nmp, 0, -1, INT_MAX, ctx->stream);
+            launch_pair_trans(djobs, nj, n_v_max, 1, nmp, 0, -1, INT_MAX, 0, ctx->stream);
             ctx->launches++;
             for (int l = 1; l <= maxL; l += 2) {
                 const int i = l >> 1, b = i & 1;
@@ -719,7 +726,7 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                     CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[b], ctx->stream));
                     CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_st[b], 0));
                     launch_pair_trans(djobs, nj, n_v_max, l + 2, nmp, (size_t)(b ^ 1) * list_buf_entries, -1, l,
-                                      ctx->aux);
+                                      0, ctx->aux);
                     CUDA_TRY(ctx, cudaEventRecord(ctx->ev_tr[b ^ 1], ctx->aux));
                     ctx->launches++;
                 }
@@ -735,12 +742,12 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                     CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[b], ctx->stream));
                     CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_st[b], 0));
                     launch_pair_trans(djobs, nj, n_v_max, l + 2, nmp, (size_t)(b ^ 1) * list_buf_entries, l + 1,
-                                      INT_MAX, ctx->aux);
+                                      INT_MAX, ctx->aux_grid_trans, ctx->aux);
                     CUDA_TRY(ctx, cudaEventRecord(ctx->ev_tr[b ^ 1], ctx->aux));
                     ctx->launches++;
                 }
                 if (l + 1 <= maxL) {
-                    launch_pair_fixup(djobs, nj, n_v_max, l + 1, nmp, ctx->stream);
+                    launch_pair_fixup(djobs, nj, n_v_max, l + 1, nmp, ctx->aux_grid_fix, ctx->stream);
                     ctx->launches++;
                 }
             }

@@ -97,8 +97,8 @@ size_t pair_entry_bytes();
 int pair_nsl(int np, int nmp);
 bool pair_supported(int P, int nmp, int n_v, int max_L);
 void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int fix_slab,
-                       int unv_from, cudaStream_t s);
-void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, cudaStream_t s);
+                       int unv_from, int max_grid, cudaStream_t s);
+void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, int max_grid, cudaStream_t s);
 void launch_pair_step(const int2 *tdesc, int n_tiles, const void *lists, size_t buf_off, int cap, int nmp, int np,
                       int nsl, int grid, unsigned long long *prof, cudaStream_t s);
 int pair_blocks_per_sm(int nmp, int np, int nsl);

@@ -130,9 +130,6 @@ constexpr int kPairHdr = 2;                      // header entries at the head o
 #ifndef MP_PAIR_L2PF
 #define MP_PAIR_L2PF 3                                     // list entries prefetched into L2, in producer rounds
 #endif
-#ifndef MP_PAIR_LOG
-#define MP_PAIR_LOG 0                                      // one shared entry log scanned by every row (vs per-row queues)
-#endif
 #ifndef MP_PAIR_ONEROW
 #define MP_PAIR_ONEROW 1                                   // one processor row per thread for tiles of <= 32
 #endif
@@ -343,13 +340,20 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
 #define MP_TRANS_MINB 8
 #endif
 __global__ void __launch_bounds__(128, MP_TRANS_MINB) pair_trans_kernel(const Job *jobs, int l, int nmp, size_t buf_off,
-                                                         int fix_slab, int unv_from) {
+                                                         int fix_slab, int unv_from, int xb, int n_items) {
+    // block item = (job, group of 4 v-tiles); a grid of n_items blocks takes one item each,
+    // a smaller (persistent) grid loops over them so that the fixup kernel's blocks can run
+    // beside it
     __shared__ Job sJ;
-    if (threadIdx.x < sizeof(Job) / 8)
-        reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
-            __ldg(reinterpret_cast<const uint64_t *>(jobs + blockIdx.y) + threadIdx.x);
-    __syncthreads();
-    pair_trans_body(sJ, blockIdx.x * 4 + (threadIdx.x >> 5), threadIdx.x & 31, l, nmp, buf_off, fix_slab, unv_from);
+    for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+        const int job = it / xb, bx = it - job * xb;
+        __syncthreads();
+        if (threadIdx.x < sizeof(Job) / 8)
+            reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
+                __ldg(reinterpret_cast<const uint64_t *>(jobs + job) + threadIdx.x);
+        __syncthreads();
+        pair_trans_body(sJ, bx * 4 + (threadIdx.x >> 5), threadIdx.x & 31, l, nmp, buf_off, fix_slab, unv_from);
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -508,19 +512,8 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     __shared__ __align__(8) uint64_t full[kPairSlotsMax];
     __shared__ __align__(8) uint64_t empty[kPairSlotsMax];
     __shared__ __align__(16) PairMeta meta[kPairSlotsMax];
-#if MP_PAIR_LOG
-    // one entry log for all rows: slot | parity << 6 | control << 7 | n_m << 8 | two rows << 12 |
-    // wrap bit << 13 | row mask << 16; each row scans it and takes the entries of its mask bit.
-    // The row codes (d, nf) travel in the slot's metadata, ordered by the full barrier.
-    static_assert(kPairProd == 1 && kPairRows <= 8, "entry log: one producer, <= 8 rows");
-    constexpr int LN = 256;                                // log entries (> round + publish interval)
-    __shared__ uint32_t lw[LN];
-    __shared__ int rpos[kPairRows];                        // log position each row has scanned (every 8)
-    uint32_t (*rq)[kPairRows][QN] = nullptr;               // (per-row queues unused)
-#else
     // per-row queues: slot | parity << 6 | control << 7 | n_m << 8 | two rows << 12 | code << 16 | wrap bit << 31
     __shared__ uint32_t rq[kPairProd][kPairRows][QN];
-#endif
     __shared__ __align__(128) PairEntry stage[kPairProd][2][kPairStage];   // list heads of this and the next tile
     __shared__ __align__(8) uint64_t stbar[kPairProd][2];
 
@@ -540,12 +533,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-#if MP_PAIR_LOG
-    for (int i = tid; i < LN; i += blockDim.x) lw[i] = 0u;
-    if (tid < kPairRows) rpos[tid] = 0;
-#else
     for (int i = tid; i < kPairProd * kPairRows * QN; i += blockDim.x) (&rq[0][0][0])[i] = 0u;
-#endif
     __syncthreads();
 
     if (warp >= kPairRows) {
@@ -557,29 +545,6 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
 #pragma unroll
         for (int rr = 0; rr < kPairRows; rr++) tails[rr] = 0;
         const unsigned lt = (1u << lane) - 1u;
-#if MP_PAIR_LOG
-        const uint32_t lw_s = smem_u32(&lw[0]);
-        int wpos = 0;                                      // log entries written
-        auto push = [&](bool act, uint32_t mask, uint32_t ent, uint64_t, uint64_t) {
-            // the active lanes are a prefix 0..cnt-1; their entries take log positions wpos..
-            const int cnt = __popc(__ballot_sync(0xffffffffu, act));
-            if (lane < kPairRows) {                        // flow control: every row has scanned pos - LN
-                int rp;
-                asm volatile("ld.volatile.shared::cta.u32 %0, [%1];" : "=r"(rp) : "r"(smem_u32(&rpos[lane])));
-                while (rp + LN < wpos + cnt) {
-                    __nanosleep(64);
-                    asm volatile("ld.volatile.shared::cta.u32 %0, [%1];" : "=r"(rp) : "r"(smem_u32(&rpos[lane])));
-                }
-            }
-            __syncwarp();
-            if (act) {
-                const int pos = wpos + lane;
-                st_entry_s(lw_s + 4u * (uint32_t)(pos & (LN - 1)),
-                           ent | mask << 16 | (uint32_t)(((pos / LN) & 1) ^ 1) << 13);
-            }
-            wpos += cnt;
-        };
-#else
         const uint32_t rq_s = smem_u32(&rq[pw][0][0]);     // shared address of this producer's queues
         auto push = [&](bool act, uint32_t mask, uint32_t ent, uint64_t codes, uint64_t codes_hi) {   // byte rr = row rr
             // append ent (+ the row's code, + the wrap bit of its position) to the queue of
@@ -601,7 +566,6 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             for (int rr = 0; rr < kPairRows; rr++)
                 if ((bal[rr] >> lane) & 1u) st_entry_s(addr[rr], word[rr]);
         };
-#endif
         // prof (MADPIPE_PROF=1): [0] producer cycles, [1] empty-barrier waits (max over lanes),
         // [2] tile setup (header), [3] consumer cycles, [4] queue waits, [5] full waits, [6] data
         // slots consumed (row visits), [7] tiles
@@ -691,9 +655,6 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                         static_assert(kPairRows == 8 || kPairRows == 16, "codes packing");
                         codes = *reinterpret_cast<const uint64_t *>(cur.code);
                         if (kPairRows > 8) codes_hi = *reinterpret_cast<const uint64_t *>(cur.code + 8);
-#if MP_PAIR_LOG
-                        *reinterpret_cast<uint64_t *>(M.e.code) = codes;   // rows' (d, nf), behind the full barrier
-#endif
                         // rows that do not read the slot release it now
                         if (__popc(mask) < kPairRows) mbar_arrive_cnt(empty0 + 8 * s, kPairRows - __popc(mask));
                         mbar_arrive_expect_tx(full0 + 8 * s, seg_bytes);
@@ -772,20 +733,6 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
         // an empty queue (the entry still carries the previous wrap's bit): back off
         // instead of spinning (a spinning warp takes issue slots from the producer and
         // the working rows)
-#if MP_PAIR_LOG
-        const uint32_t want = (uint32_t)(((head[0] / LN) & 1) ^ 1);
-        const uint32_t *qe = &lw[head[0] & (LN - 1)];
-        uint32_t ent;
-        while (((ent = ld_entry(qe)) >> 13 & 1u) != want) {
-#if MP_POLL_NS > 0
-            __nanosleep(MP_POLL_NS);
-#endif
-        }
-        head[0]++;
-        if ((head[0] & 7) == 0 && lane == 0)               // publish the scan position (flow control)
-            asm volatile("st.volatile.shared::cta.u32 [%0], %1;" ::"r"(smem_u32(&rpos[r])), "r"(head[0]));
-        if (!((ent >> (16 + r)) & 1u)) continue;           // not this row's entry
-#else
         const uint32_t want = (uint32_t)(((head[qp] / QN) & 1) ^ 1);
         const uint32_t *qe = &rq[qp][r][head[qp] & (QN - 1)];
         uint32_t ent;
@@ -795,7 +742,6 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
 #endif
         }
         head[qp]++;
-#endif
         const int s = (int)(ent & 63u);                    // this row's slot
         const long long tb = prof ? clock64() : 0;
         mbar_wait(full0 + 8 * s, (ent >> 6) & 1u);
@@ -831,14 +777,8 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
         } else {
             // rows lane and lane+32 are relaxed whether or not they exist in this tile
             // (np < 64): the extra rows read in-bounds ring bytes and are never stored
-#if MP_PAIR_LOG
-            const uint32_t code = M.e.code[r];
-            const int d = (int)(code & 127u);
-            const bool nf = (code >> 7) & 1u;
-#else
             const int d = (int)((ent >> 16) & 127u);
             const bool nf = (ent >> 23) & 1u;
-#endif
             const double U = isB ? M.e.U1 : M.e.U0;
             const int lim = (int)((ent >> 8) & 15u) - 1 - d;   // n_m - 1 - d
             const char *slot = ring + s * seg_bytes;
@@ -918,13 +858,18 @@ __device__ __forceinline__ void pair_fixup_body(const Job &J, int v, int lane, i
 #ifndef MP_FIX_MINB
 #define MP_FIX_MINB 1
 #endif
-__global__ void __launch_bounds__(128, MP_FIX_MINB) pair_fixup_kernel(const Job *jobs, int l1, int nmp) {
+__global__ void __launch_bounds__(128, MP_FIX_MINB) pair_fixup_kernel(const Job *jobs, int l1, int nmp, int xb,
+                                                                       int n_items) {
     __shared__ Job sJ;
-    if (threadIdx.x < sizeof(Job) / 8)
-        reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
-            __ldg(reinterpret_cast<const uint64_t *>(jobs + blockIdx.y) + threadIdx.x);
-    __syncthreads();
-    pair_fixup_body(sJ, blockIdx.x * 4 + (threadIdx.x >> 5), threadIdx.x & 31, l1, nmp);
+    for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+        const int job = it / xb, bx = it - job * xb;
+        __syncthreads();
+        if (threadIdx.x < sizeof(Job) / 8)
+            reinterpret_cast<uint64_t *>(&sJ)[threadIdx.x] =
+                __ldg(reinterpret_cast<const uint64_t *>(jobs + job) + threadIdx.x);
+        __syncthreads();
+        pair_fixup_body(sJ, bx * 4 + (threadIdx.x >> 5), threadIdx.x & 31, l1, nmp);
+    }
 }
 
 
@@ -954,13 +899,17 @@ bool pair_supported(int P, int nmp, int n_v, int max_L) {
 }
 
 void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp, size_t buf_off, int fix_slab,
-                       int unv_from, cudaStream_t s) {
+                       int unv_from, int max_grid, cudaStream_t s) {
     const int nvt = (n_v_max + kPairVB - 1) / kPairVB + kPairE;
-    pair_trans_kernel<<<dim3((nvt + 3) / 4, n_jobs), 128, 0, s>>>(jobs, l, nmp, buf_off, fix_slab, unv_from);
+    const int xb = (nvt + 3) / 4, items = xb * n_jobs;
+    const int grid = max_grid > 0 && max_grid < items ? max_grid : items;
+    pair_trans_kernel<<<grid, 128, 0, s>>>(jobs, l, nmp, buf_off, fix_slab, unv_from, xb, items);
 }
 
-void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, cudaStream_t s) {
-    pair_fixup_kernel<<<dim3((n_v_max + 3) / 4, n_jobs), 128, 0, s>>>(jobs, l1, nmp);
+void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, int max_grid, cudaStream_t s) {
+    const int xb = (n_v_max + 3) / 4, items = xb * n_jobs;
+    const int grid = max_grid > 0 && max_grid < items ? max_grid : items;
+    pair_fixup_kernel<<<grid, 128, 0, s>>>(jobs, l1, nmp, xb, items);
 }
 
 static int pair_round(int nsl) {

@@ -23,7 +23,6 @@ VARIANTS = {
     "l2pf2": "-DMP_PAIR_L2PF=2",
     "l2pf4": "-DMP_PAIR_L2PF=4",
     "ctas3": "-DMP_PAIR_CTAS=3",                  # 3 CTAs per SM (16-slot rings, <= 75 registers)
-    "log": "-DMP_PAIR_LOG=1",                     # one entry log scanned by every row instead of per-row queues
 }
 
 if __name__ == "__main__":
