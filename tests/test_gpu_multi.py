@@ -171,3 +171,18 @@ def test_batch_sweep_ranks_then_resolve_equals_world1(ctx, nctx, world):
             assert i not in got
     for g, rr in zip(nctx.solve_batch(chains, Ps, Ms, Bs, *d), ref):
         _same(g, rr)
+
+
+def test_fig6_sweep_batch_matches_oracle(ctx):
+    """NEXT row f4 (scripts/fig6_sweep.py): the 84 Fig. 6-style instances -- ResNet-50-shaped
+    chain, M = 3..16 GB x P in {2, 4, 8} x beta in {12, 24} GB/s, the paper's 11 x 51
+    discretisation -- in one madpipe_solve_batch, each equal to the oracle."""
+    ch = chaingen.resnet50()
+    inst = [(g * 10**9, P, b) for b in (12e9, 24e9) for P in (2, 4, 8) for g in range(3, 17)]
+    n_c = 48
+    res = ctx.solve_batch([ch] * len(inst), [P for _, P, _ in inst], [M for M, _, _ in inst],
+                          [b for _, _, b in inst], 11, 51, n_c)
+    for (M, P, b), got in zip(inst, res):
+        ref = oracle.solve(ch, P, M, b, 11, 51, n_c, early_exit=True, n_threads=8)
+        _same(got, ref)
+        _verify(ch, P, M, b, got)
