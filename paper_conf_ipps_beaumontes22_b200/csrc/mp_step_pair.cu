@@ -579,8 +579,10 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             mbar_arrive_expect_tx(st0 + 8 * buf, stage_bytes);
             bulk_g2s(smem_u32(&stage[pw][buf][0]), lists + dsc.x, stage_bytes, st0 + 8 * buf);
         };
-        const int G = (int)gridDim.x * kPairProd;           // tile stride of this producer
-        const int t0 = (int)blockIdx.x + pw * (int)gridDim.x;
+        // with two producers both walk the same tiles and split each tile's entries (producer
+        // pw takes entries pw, pw + 2, ...), each ending its share with a tile-end marker
+        const int G = (int)gridDim.x;                       // tile stride
+        const int t0 = (int)blockIdx.x;
         int2 desc = t0 < n_tiles ? __ldg(tdesc + t0) : make_int2(0, 0);
         int2 nextd = t0 + G < n_tiles ? __ldg(tdesc + t0 + G) : make_int2(0, 0);
         if (lane == 0 && t0 < n_tiles) stage_copy(desc, 0);
@@ -605,26 +607,28 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             // the tiles' ends in turn)
             const bool skip = hd.n < 0 || np <= 0;
             // first round's entries
+            const int n_all = skip ? 0 : hd.n;
+            const int n = (n_all - pw + kPairProd - 1) / kPairProd;   // this producer's share of the entries
+            auto gidx = [&](int q_) { return q_ * kPairProd + pw; };   // share index -> list index
             PairEntry cur;
-            if (!skip && lane < round) cur = entry(lane);
+            if (n > 0 && lane < round && lane < n) cur = entry(gidx(lane));
             const int64_t rowlen = (int64_t)hd.P * NMP;
             const int64_t slab = (int64_t)hd.n_v * rowlen;
             const uint32_t seg_bytes = (uint32_t)(np + 1) * NMP * 8u;
-            const int n = skip ? 0 : hd.n;
             const int stages = n + 1;                      // entries, then the tile-end marker
             if (prof) { t_set += clock64() - t_t0; n_tl++; }
             for (int r0 = 0; r0 < stages; r0 += round) {
                 const int q = r0 + lane;
                 const bool act = lane < round && q < stages;
                 PairEntry nxt;                             // prefetch the next round's entry
-                if (lane < round && q + round < n) nxt = entry(q + round);
+                if (lane < round && q + round < n) nxt = entry(gidx(q + round));
 #if MP_PAIR_L2PF
                 // and pull entries MP_PAIR_L2PF rounds ahead into L2 (lists beyond the staged head
                 // are read from global memory; a DRAM miss there stalls the whole pipeline)
                 {
                     const int qf = q + MP_PAIR_L2PF * round;
-                    if (lane < round && qf < n && qf + kPairHdr >= stage_n)
-                        asm volatile("prefetch.global.L2 [%0];" ::"l"(tl + kPairHdr + qf));
+                    if (lane < round && qf < n && gidx(qf) + kPairHdr >= stage_n)
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(tl + kPairHdr + gidx(qf)));
                 }
 #endif
                 uint32_t mask = 0, ent = 0;
@@ -749,7 +753,9 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
         const PairMeta &M = meta[s];
         if (ent & 128u) {                                  // control slot (tile end / terminate)
         const int flags = M.flags;
-        if (flags & 4) {
+        if ((flags & 4) && kPairProd > 1 && qp < kPairProd - 1) {
+            qp++;                                          // the other producer's terminate follows
+        } else if (flags & 4) {
             if (prof && lane == 0) {
                 atomicAdd(prof + 3, (unsigned long long)(clock64() - t_c0));
                 atomicAdd(prof + 4, (unsigned long long)t_q);
@@ -758,7 +764,9 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             }
             break;
         }
-        if (flags & 1) {                                   // tile end: clamp (Q12), store, flag
+        else if ((flags & 1) && kPairProd > 1 && qp < kPairProd - 1) {
+            qp++;                                          // end of one producer's share of the tile
+        } else if (flags & 1) {                            // tile end: clamp (Q12), store, flag
             const int np = M.np, n_m = M.n_m;
             const int v = isB ? M.t.v0B + (r - kPairVB) : M.t.v0A + r;
             const bool ok = !(flags & 16) && (!isB || M.hasB) && v >= 0 && v < M.n_v;   // 16: empty tile
@@ -772,7 +780,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 atomicOr(M.t.flA + (isB ? M.n_v : 0) + v, 1u);
 #pragma unroll
             for (int i = 0; i < NMP; i++) { b0[i] = MP_INF; b1[i] = MP_INF; }
-            if (kPairProd > 1) qp = (qp + 1) % kPairProd;   // the next tile comes from the next producer
+            qp = 0;                                        // the next tile starts with producer 0's share
         }
         } else {
             // rows lane and lane+32 are relaxed whether or not they exist in this tile

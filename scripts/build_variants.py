@@ -23,6 +23,7 @@ VARIANTS = {
     "l2pf2": "-DMP_PAIR_L2PF=2",
     "l2pf4": "-DMP_PAIR_L2PF=4",
     "ctas3": "-DMP_PAIR_CTAS=3",                  # 3 CTAs per SM (16-slot rings, <= 75 registers)
+    "prod2": "-DMP_PAIR_NPROD=2",                 # two producer warps per CTA splitting each tile's entries
 }
 
 if __name__ == "__main__":
