@@ -474,7 +474,11 @@ def main():
         "effective_updates_per_step": eff_step,
         "effective_updates_per_s": eff_step * K / (tot_ms / 1e3),
         "useful_updates_per_step": useful_step,
-        "result": main_run["summ"],
+        "result": dict(main_run["summ"], **(
+            {"oracle_cand_index_sum": sum(c["oracle_cand_index"] for c in cfg["chains"]),
+             "matches_oracle": main_run["summ"]["cand_index_sum"] == sum(c["oracle_cand_index"] for c in cfg["chains"])}
+            if batch else {"oracle_cand_index": cfg.get("oracle_cand_index"),
+                           "matches_oracle": main_run["summ"]["cand_index"] == cfg.get("oracle_cand_index")})),
         "roofline": roof,
         "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(), "cpu_baseline": cpu,
     }
