@@ -555,7 +555,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     #pragma unroll
         for (int rr = 0; rr < kPairRows; rr++) tails[rr] = 0;
         const unsigned lt = (1u << lane) - 1u;
-        const uint32_t rq_s = smem_u32(&rq[warp > kPairRows && !kPairPusher ? warp - kPairRows : 0][0][0]);   // this producer's queues
+        const uint32_t rq_s = smem_u32(&rq[0][0][0]);       // the (one) producer's queues
         auto push = [&](bool act, uint32_t mask, uint32_t ent, uint64_t codes, uint64_t codes_hi) {   // byte rr = row rr
             // append ent (+ the row's code, + the wrap bit of its position) to the queue of
             // every row in mask, in lane order.  All ballots first, then the positions and
@@ -596,7 +596,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     #pragma unroll
         for (int rr = 0; rr < kPairRows; rr++) tails[rr] = 0;
         const unsigned lt = (1u << lane) - 1u;
-        const uint32_t rq_s = smem_u32(&rq[warp > kPairRows && !kPairPusher ? warp - kPairRows : 0][0][0]);   // this producer's queues
+        const uint32_t rq_s = smem_u32(&rq[pw][0][0]);      // this producer's queues
         auto push = [&](bool act, uint32_t mask, uint32_t ent, uint64_t codes, uint64_t codes_hi) {   // byte rr = row rr
             // append ent (+ the row's code, + the wrap bit of its position) to the queue of
             // every row in mask, in lane order.  All ballots first, then the positions and
