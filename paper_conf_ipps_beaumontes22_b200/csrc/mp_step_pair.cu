@@ -119,12 +119,7 @@ constexpr int kPairSlotsMax = kPairVB > 4 ? 48 : 32;  // ring slots (6-bit slot 
 #endif
 constexpr int kPairProd = MP_PAIR_NPROD;         // producer warps: producer p takes the CTA's tiles p, p+2, ..
                                                  // with its own half of the ring and its own row queues
-#ifndef MP_PAIR_PUSHER
-#define MP_PAIR_PUSHER 0
-#endif
-constexpr int kPairPusher = MP_PAIR_PUSHER;      // 1: a second warp does the producer's queue pushes
-static_assert(kPairPusher == 0 || kPairProd == 1, "pusher warp: one producer");
-constexpr int kPairThreads = 32 * (kPairRows + kPairProd + kPairPusher);
+constexpr int kPairThreads = 32 * (kPairRows + kPairProd);
 constexpr int kPairHdr = 2;                      // header entries at the head of each tile list
 #ifndef MP_POLL_NS
 #define MP_POLL_NS 250
@@ -521,10 +516,6 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
     __shared__ uint32_t rq[kPairProd][kPairRows][QN];
     __shared__ __align__(128) PairEntry stage[kPairProd][2][kPairStage];   // list heads of this and the next tile
     __shared__ __align__(8) uint64_t stbar[kPairProd][2];
-    // producer -> pusher handoff (kPairPusher): per lane {ent, mask, codes lo, codes hi}, double-buffered
-    __shared__ uint4 pbuf[kPairPusher ? 2 : 1][32];
-    __shared__ uint32_t pfin[2];
-    __shared__ __align__(8) uint64_t pbar[4];              // full[2], empty[2]
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
@@ -540,72 +531,30 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             mbar_init(smem_u32(&stbar[p][0]), 1);
             mbar_init(smem_u32(&stbar[p][1]), 1);
         }
-        for (int i = 0; i < 4; i++) mbar_init(smem_u32(&pbar[i]), 32);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     for (int i = tid; i < kPairProd * kPairRows * QN; i += blockDim.x) (&rq[0][0][0])[i] = 0u;
     __syncthreads();
 
-    const uint32_t pfull0 = smem_u32(&pbar[0]), pempty0 = smem_u32(&pbar[2]);
-    if (kPairPusher && warp == kPairRows + kPairProd) {
-        // =========================================================== pusher warp
-        // takes each producer round {ent, mask, codes} from the handoff buffer and appends it
-        // to the row queues, while the producer prepares the next round
-        int tails[kPairRows];                              // entries pushed per row (same in every lane)
-    #pragma unroll
-        for (int rr = 0; rr < kPairRows; rr++) tails[rr] = 0;
-        const unsigned lt = (1u << lane) - 1u;
-        const uint32_t rq_s = smem_u32(&rq[0][0][0]);       // the (one) producer's queues
-        auto push = [&](bool act, uint32_t mask, uint32_t ent, uint64_t codes, uint64_t codes_hi) {   // byte rr = row rr
-            // append ent (+ the row's code, + the wrap bit of its position) to the queue of
-            // every row in mask, in lane order.  All ballots first, then the positions and
-            // words, then the stores: independent work the scheduler can overlap.
-            unsigned bal[kPairRows];
-    #pragma unroll
-            for (int rr = 0; rr < kPairRows; rr++) bal[rr] = __ballot_sync(0xffffffffu, act && ((mask >> rr) & 1u));
-            uint32_t addr[kPairRows], word[kPairRows];
-    #pragma unroll
-            for (int rr = 0; rr < kPairRows; rr++) {
-                const int pos = tails[rr] + __popc(bal[rr] & lt);
-                const uint64_t cw = rr < 8 ? codes : codes_hi;
-                addr[rr] = rq_s + 4u * (uint32_t)(rr * QN + (pos & (QN - 1)));
-                word[rr] = ent | (uint32_t)((cw >> (8 * (rr & 7))) & 0xFFu) << 16 | (uint32_t)(((pos / QN) & 1) ^ 1) << 31;
-                tails[rr] += __popc(bal[rr]);
-            }
-    #pragma unroll
-            for (int rr = 0; rr < kPairRows; rr++)
-                if ((bal[rr] >> lane) & 1u) st_entry_s(addr[rr], word[rr]);
-        };
-        for (int u = 0;; u++) {
-            const int b = u & 1;
-            mbar_wait(pfull0 + 8 * b, (uint32_t)((u >> 1) & 1));
-            const uint4 x = pbuf[b][lane];
-            const uint32_t fin = pfin[b];
-            push(x.y != 0u, x.y, x.x, (uint64_t)x.w << 32 | x.z, 0ull);
-            mbar_arrive(pempty0 + 8 * b);
-            if (fin) break;
-        }
-        return;
-    }
     if (warp >= kPairRows) {
         // =========================================================== producer warp(s)
         const int pw = warp - kPairRows;                   // producer index
         const int nslp = nsl / kPairProd, s_base = pw * nslp;   // this producer's ring slots
         int sl = 0, wraps = 0;
         int tails[kPairRows];                              // entries pushed per row (same in every lane)
-    #pragma unroll
+#pragma unroll
         for (int rr = 0; rr < kPairRows; rr++) tails[rr] = 0;
         const unsigned lt = (1u << lane) - 1u;
-        const uint32_t rq_s = smem_u32(&rq[pw][0][0]);      // this producer's queues
+        const uint32_t rq_s = smem_u32(&rq[pw][0][0]);     // shared address of this producer's queues
         auto push = [&](bool act, uint32_t mask, uint32_t ent, uint64_t codes, uint64_t codes_hi) {   // byte rr = row rr
             // append ent (+ the row's code, + the wrap bit of its position) to the queue of
             // every row in mask, in lane order.  All ballots first, then the positions and
             // words, then the stores: independent work the scheduler can overlap.
             unsigned bal[kPairRows];
-    #pragma unroll
+#pragma unroll
             for (int rr = 0; rr < kPairRows; rr++) bal[rr] = __ballot_sync(0xffffffffu, act && ((mask >> rr) & 1u));
             uint32_t addr[kPairRows], word[kPairRows];
-    #pragma unroll
+#pragma unroll
             for (int rr = 0; rr < kPairRows; rr++) {
                 const int pos = tails[rr] + __popc(bal[rr] & lt);
                 const uint64_t cw = rr < 8 ? codes : codes_hi;
@@ -613,7 +562,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 word[rr] = ent | (uint32_t)((cw >> (8 * (rr & 7))) & 0xFFu) << 16 | (uint32_t)(((pos / QN) & 1) ^ 1) << 31;
                 tails[rr] += __popc(bal[rr]);
             }
-    #pragma unroll
+#pragma unroll
             for (int rr = 0; rr < kPairRows; rr++)
                 if ((bal[rr] >> lane) & 1u) st_entry_s(addr[rr], word[rr]);
         };
@@ -621,16 +570,6 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
         // [2] tile setup (header), [3] consumer cycles, [4] queue waits, [5] full waits, [6] data
         // slots consumed (row visits), [7] tiles
         long long t_p0 = clock64(), t_we = 0, t_set = 0, n_tl = 0, t_push = 0;
-        int hu = 0;                                        // handoff rounds (kPairPusher)
-        auto handoff = [&](bool act, uint32_t mask, uint32_t ent, uint64_t codes, bool fin) {
-            // hand the round to the pusher warp (kPairPusher)
-            const int b = hu & 1;
-            if (hu >= 2) mbar_wait(pempty0 + 8 * b, (uint32_t)(((hu >> 1) - 1) & 1));
-            pbuf[b][lane] = make_uint4(ent, act ? mask : 0u, (uint32_t)codes, (uint32_t)(codes >> 32));
-            if (lane == 0) pfin[b] = fin ? 1u : 0u;
-            mbar_arrive(pfull0 + 8 * b);
-            hu++;
-        };
         // the head of each tile's list (header + first entries) is bulk-copied into a
         // staging buffer one tile ahead, so a tile starts without a global-load round trip
         const uint32_t st0 = smem_u32(&stbar[pw][0]);
@@ -742,8 +681,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                     }
                 }
                 const long long tpu = prof ? clock64() : 0;
-                if (kPairPusher) handoff(act, mask, ent, codes, false);
-                else push(act, mask, ent, codes, codes_hi);
+                push(act, mask, ent, codes, codes_hi);
                 if (prof && lane == 0) t_push += clock64() - tpu;
                 cur = nxt;
                 const int adv = min(round, stages - r0);
@@ -761,8 +699,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                 ent = (uint32_t)sg_ | (uint32_t)(wraps & 1) << 6 | 128u;   // control slot
                 mbar_arrive(full0 + 8 * sg_);
             }
-            if (kPairPusher) handoff(act, (1u << kPairRows) - 1u, ent, 0ull, true);
-            else push(act, (1u << kPairRows) - 1u, ent, 0ull, 0ull);
+            push(act, (1u << kPairRows) - 1u, ent, 0ull, 0ull);
         }
         if (prof && lane == 0) {
             atomicAdd(prof + 0, (unsigned long long)(clock64() - t_p0));

@@ -24,7 +24,6 @@ VARIANTS = {
     "l2pf4": "-DMP_PAIR_L2PF=4",
     "ctas3": "-DMP_PAIR_CTAS=3",                  # 3 CTAs per SM (16-slot rings, <= 75 registers)
     "prod2": "-DMP_PAIR_NPROD=2",                 # two producer warps per CTA splitting each tile's entries
-    "pusher": "-DMP_PAIR_PUSHER=1",               # a pusher warp appends the producer's rounds to the row queues
 }
 
 if __name__ == "__main__":
