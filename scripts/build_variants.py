@@ -17,6 +17,7 @@ VARIANTS = {
     "qatomic": "-DMP_QUEUE_ATOMIC=1",             # queue words through shared atomics (racecheck-clean)
     "noprof": "-DMP_PAIR_PROF=0",                 # cycle counters compiled out
     "poll0": "-DMP_POLL_NS=0",                    # consumers spin without back-off
+    "poll100": "-DMP_POLL_NS=100",
     "tworow": "-DMP_PAIR_ONEROW=0",               # always relax both processor rows of a thread
     "nol2pf": "-DMP_PAIR_L2PF=0",                 # no L2 prefetch of list entries ahead of the producer
     "l2pf6": "-DMP_PAIR_L2PF=6",                  # L2 prefetch 6 rounds ahead
