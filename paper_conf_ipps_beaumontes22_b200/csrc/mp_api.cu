@@ -66,6 +66,7 @@ struct madpipe_ctx {
     // MADPIPE_AUX_GRID=t,f: persistent grids of t and f blocks per SM for the pair path's list
     // builder and fixup kernels (they run side by side on two streams; 0 = one block per item)
     int aux_grid_trans = 0, aux_grid_fix = 0;
+    int replay_pass = -1, replay_reps = 0, replay_diag = 0;   // MADPIPE_REPLAY=pass,reps,diag (diagnostic)
     int trans_overlap = 0;    // MADPIPE_TRANS_OVERLAP=1: pair path builds pass i+1's lists beside step(i) (measured
                               // slower at GPT: 909 vs 886 ms, 5% more entries kept unverified + contention)
     DevBuf profbuf;
@@ -279,6 +280,7 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, int32_t rank, i
     if (const char *e = getenv("MADPIPE_NPROD")) c->n_prod = std::max(1, std::min(4, atoi(e)));
     if (const char *e = getenv("MADPIPE_TILE_BLOCK")) c->tile_block = std::max(1, atoi(e));
     if (const char *e = getenv("MADPIPE_TRANS_OVERLAP")) c->trans_overlap = atoi(e) != 0;
+    if (const char *e = getenv("MADPIPE_REPLAY")) sscanf(e, "%d,%d,%d", &c->replay_pass, &c->replay_reps, &c->replay_diag);
     if (const char *e = getenv("MADPIPE_AUX_GRID")) {
         int t = 0, f = 0;
         if (sscanf(e, "%d,%d", &t, &f) == 2) { c->aux_grid_trans = t * c->num_sms; c->aux_grid_fix = f * c->num_sms; }
@@ -729,6 +731,27 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                                       0, ctx->aux);
                     CUDA_TRY(ctx, cudaEventRecord(ctx->ev_tr[b ^ 1], ctx->aux));
                     ctx->launches++;
+                }
+                if (i == ctx->replay_pass && ctx->replay_reps > 0) {
+                    // diagnostic (MADPIPE_REPLAY=pass,reps,diag): this pass's step kernel
+                    // re-launched on the same lists (it reads slabs <= l-1 and writes l, l+1: idempotent)
+                    // and timed alone; with an MP_DIAG=1 build, diag bit 0 drops the relaxation and bit 1
+                    // the copies in the re-launches only
+                    cudaEvent_t e0, e1;
+                    cudaEventCreate(&e0);
+                    cudaEventCreate(&e1);
+                    cudaEventRecord(e0, ctx->stream);
+                    for (int rp = 0; rp < ctx->replay_reps; rp++)
+                        launch_pair_step((const int2 *)ctx->tdesc.p, n_tiles, ctx->tlist.p, b * list_buf_entries, cap,
+                                         nmp, p_np, nsg, persist_grid, nullptr, ctx->stream, ctx->replay_diag);
+                    cudaEventRecord(e1, ctx->stream);
+                    cudaEventSynchronize(e1);
+                    float ms = 0.f;
+                    cudaEventElapsedTime(&ms, e0, e1);
+                    fprintf(stderr, "[madpipe replay] pass %d, diag %d, %d jobs, %d tiles: %.4f ms per step launch\n", i,
+                            ctx->replay_diag, nj, n_tiles, ms / ctx->replay_reps);
+                    cudaEventDestroy(e0);
+                    cudaEventDestroy(e1);
                 }
                 if (per_launch) cudaEventRecord(ctx->ev_pool[2 * n_rec], ctx->stream);
                 launch_pair_step((const int2 *)ctx->tdesc.p, n_tiles, ctx->tlist.p, b * list_buf_entries, cap, nmp,

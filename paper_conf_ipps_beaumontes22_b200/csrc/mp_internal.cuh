@@ -100,7 +100,7 @@ void launch_pair_trans(const Job *jobs, int n_jobs, int n_v_max, int l, int nmp,
                        int unv_from, int max_grid, cudaStream_t s);
 void launch_pair_fixup(const Job *jobs, int n_jobs, int n_v_max, int l1, int nmp, int max_grid, cudaStream_t s);
 void launch_pair_step(const int2 *tdesc, int n_tiles, const void *lists, size_t buf_off, int cap, int nmp, int np,
-                      int nsl, int grid, unsigned long long *prof, cudaStream_t s);
+                      int nsl, int grid, unsigned long long *prof, cudaStream_t s, int diag = 0);
 int pair_blocks_per_sm(int nmp, int np, int nsl);
 int persist_blocks_per_sm(int nmp, int np, int vb, int nsg, int n_prod);
 void persist_geom(int P, int n_v, int nmp, int *vb, int *np, int *n_ptiles, int *n_tiles);

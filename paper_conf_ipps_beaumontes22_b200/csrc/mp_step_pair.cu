@@ -133,6 +133,10 @@ constexpr int kPairHdr = 2;                      // header entries at the head o
 #ifndef MP_PAIR_ONEROW
 #define MP_PAIR_ONEROW 1                                   // one processor row per thread for tiles of <= 32
 #endif
+#ifndef MP_DIAG
+#define MP_DIAG 0                                          // 1: the `diag` launch argument is honoured (diagnostic
+#endif                                                     // replays only, wrong results): bit 0 = consumers skip
+                                                           // the relaxation, bit 1 = producer skips the copies
 #ifndef MP_PAIR_STAGE
 #define MP_PAIR_STAGE 32
 #endif
@@ -496,7 +500,11 @@ template <int NMP>
 __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(const int2 *__restrict__ tdesc, int n_tiles,
                                                                     const PairEntry *__restrict__ lists,
                                                                     int np_max, int nsl, int round,
-                                                                    int stage_n, unsigned long long *prof) {
+                                                                    int stage_n, unsigned long long *prof,
+                                                                    int diag) {
+#if !MP_DIAG
+    diag = 0;                                              // MADPIPE_REPLAY diagnostics compiled out
+#endif
     // Slots are shared by the rows that read them: the producer pushes each slot
     // (with the parity of its full-barrier phase) into the queue of every row in
     // its mask; a row warp visits only its own slots; the last reader (reference
@@ -649,10 +657,11 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                     ent = (uint32_t)s | (uint32_t)(use & 1) << 6 | (uint32_t)hd.n_m << 8 | (np > 32 || !MP_PAIR_ONEROW ? 4096u : 0u);
                     PairMeta &M = meta[s];
                     if (q < n) {
-                        bulk_g2s(ring_s + 8u * (uint32_t)(s * seg_doubles),
-                                 hd.table + (int64_t)(cur.k - 1) * slab + (int64_t)cur.vp * rowlen +
-                                     (int64_t)(p_lo - 1) * NMP,
-                                 seg_bytes, full0 + 8 * s);
+                        if (!(diag & 2))
+                            bulk_g2s(ring_s + 8u * (uint32_t)(s * seg_doubles),
+                                     hd.table + (int64_t)(cur.k - 1) * slab + (int64_t)cur.vp * rowlen +
+                                         (int64_t)(p_lo - 1) * NMP,
+                                     seg_bytes, full0 + 8 * s);
                         mask = cur.mask;
                         M.e.U0 = cur.U0;
                         M.e.U1 = cur.U1;
@@ -661,7 +670,8 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                         if (kPairRows > 8) codes_hi = *reinterpret_cast<const uint64_t *>(cur.code + 8);
                         // rows that do not read the slot release it now
                         if (__popc(mask) < kPairRows) mbar_arrive_cnt(empty0 + 8 * s, kPairRows - __popc(mask));
-                        mbar_arrive_expect_tx(full0 + 8 * s, seg_bytes);
+                        if (diag & 2) mbar_arrive(full0 + 8 * s);
+                        else mbar_arrive_expect_tx(full0 + 8 * s, seg_bytes);
                     } else {
                         mask = (1u << kPairRows) - 1u;
                         ent |= 128u;                       // control slot
@@ -790,7 +800,8 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             const double U = isB ? M.e.U1 : M.e.U0;
             const int lim = (int)((ent >> 8) & 15u) - 1 - d;   // n_m - 1 - d
             const char *slot = ring + s * seg_bytes;
-            if (ent & 4096u)                               // the tile has > 32 processor rows
+            if (diag & 1) {
+            } else if (ent & 4096u)                               // the tile has > 32 processor rows
                 pair_relax<NMP, true>(b0, b1, slot, off0, off1, m2, d, nf, U, lim);
             else
                 pair_relax<NMP, false>(b0, b1, slot, off0, off1, m2, d, nf, U, lim);
@@ -934,7 +945,7 @@ static int pair_smem(int np, int nmp, int nsl) {
 }
 
 void launch_pair_step(const int2 *tdesc, int n_tiles, const void *lists, size_t buf_off, int cap, int nmp, int np,
-                      int nsl, int grid, unsigned long long *prof, cudaStream_t s) {
+                      int nsl, int grid, unsigned long long *prof, cudaStream_t s, int diag) {
     const int smem = pair_smem(np, nmp, nsl);
     const int stage_n = cap < kPairStage ? cap : kPairStage;
     const PairEntry *L = reinterpret_cast<const PairEntry *>(lists) + buf_off;
@@ -942,7 +953,7 @@ void launch_pair_step(const int2 *tdesc, int n_tiles, const void *lists, size_t 
 #define MP_CASE(N)                                                                                     \
     case N:                                                                                            \
         cudaFuncSetAttribute(pair_step_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);   \
-        pair_step_kernel<N><<<grid, kPairThreads, smem, s>>>(tdesc, n_tiles, L, np, nsl, pair_round(nsl / kPairProd), stage_n, prof); \
+        pair_step_kernel<N><<<grid, kPairThreads, smem, s>>>(tdesc, n_tiles, L, np, nsl, pair_round(nsl / kPairProd), stage_n, prof, diag); \
         break;
         MP_CASE(4) MP_CASE(8)
 #undef MP_CASE

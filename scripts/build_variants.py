@@ -13,7 +13,6 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 VARIANTS = {
     "base": "",                                   # the defaults
-    "vb8": "-DMP_PAIR_VB=8",                      # 8 delay rows x 2 layers per tile, 1 CTA per SM
     "qatomic": "-DMP_QUEUE_ATOMIC=1",             # queue words through shared atomics (racecheck-clean)
     "noprof": "-DMP_PAIR_PROF=0",                 # cycle counters compiled out
     "poll0": "-DMP_POLL_NS=0",                    # consumers spin without back-off
@@ -24,7 +23,9 @@ VARIANTS = {
     "l2pf2": "-DMP_PAIR_L2PF=2",
     "l2pf4": "-DMP_PAIR_L2PF=4",
     "ctas3": "-DMP_PAIR_CTAS=3",                  # 3 CTAs per SM (16-slot rings, <= 75 registers)
-    "prod2": "-DMP_PAIR_NPROD=2",                 # two producer warps per CTA splitting each tile's entries
+    # MADPIPE_REPLAY=pass,reps,diag honoured (diag 1: consumers skip the relaxation, 2: producer
+    # skips the copies, 3: both) -- diagnostic replays only, never the solve itself
+    "diag": "-DMP_DIAG=1",
 }
 
 if __name__ == "__main__":
