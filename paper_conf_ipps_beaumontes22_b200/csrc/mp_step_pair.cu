@@ -125,7 +125,7 @@ constexpr int kPairHdr = 2;                      // header entries at the head o
 #define MP_POLL_NS 250
 #endif
 #ifndef MP_PAIR_PROF
-#define MP_PAIR_PROF 1                                     // MADPIPE_PROF=1 cycle counters in pair_step_kernel
+#define MP_PAIR_PROF 0                                     // 1: MADPIPE_PROF=1 cycle counters in pair_step_kernel (build variant "prof")
 #endif
 #ifndef MP_PAIR_L2PF
 #define MP_PAIR_L2PF 3                                     // list entries prefetched into L2, in producer rounds
