@@ -212,6 +212,12 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
     const int lr = isB ? l + 1 : l;              // the row's layer
     const int v = isB ? vt * kPairVB - delta + (r - kPairVB) : vt * kPairVB + r;
     const bool row_ok = (!isB || hasB) && v >= 0 && v < J.n_v;
+    if (__ballot_sync(0xffffffffu, row_ok) == 0u) {    // no output row in this tile (one of the extra v-tiles
+        if (lane == 0)                           // beyond the layer-(l+1) shift): the step kernel skips it
+            reinterpret_cast<PairHdr *>(reinterpret_cast<PairEntry *>(J.tlist) + buf_off +
+                                        (size_t)vt * J.code_cap)->n = -1;
+        return;
+    }
     const size_t rowlen = (size_t)J.P * nmp;
     const size_t slab = (size_t)J.n_v * rowlen;
     const double Ulr = J.Up[lr];
@@ -364,7 +370,7 @@ __global__ void __launch_bounds__(128, MP_TRANS_MINB) pair_trans_kernel(const Jo
 // a5 for the layer pair: the persistent two-layer step kernel.
 // ---------------------------------------------------------------------------
 struct PairMeta {
-    int16_t flags;          // 0 = data, 1 = tile end (store the rows; | 16: empty tile), 4 = terminate
+    int16_t flags;          // 0 = data, 1 = tile end (store the rows), 4 = terminate
     int16_t np;             // processor rows of the tile
     int32_t n_m;
     union {
@@ -610,12 +616,11 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
             const int pt = mine.y;
             const int p_lo = 1 + pt * np_max;
             const int np = min(np_max, hd.P - p_lo);
-            // a job with no layer l, or no processors in this tile: no entries and an empty
-            // tile end (consumers keep one tile end per tile: with two producers they take
-            // the tiles' ends in turn)
-            const bool skip = hd.n < 0 || np <= 0;
+            // a job with no layer l, a tile with no output row, or no processors in this tile:
+            // nothing to store, no slot at all
+            if (hd.n < 0 || np <= 0) continue;
             // first round's entries
-            const int n_all = skip ? 0 : hd.n;
+            const int n_all = hd.n;
             const int n = (n_all - pw + kPairProd - 1) / kPairProd;   // this producer's share of the entries
             auto gidx = [&](int q_) { return q_ * kPairProd + pw; };   // share index -> list index
             PairEntry cur;
@@ -677,7 +682,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
                         ent |= 128u;                       // control slot
                         M.np = (int16_t)np;
                         M.n_m = hd.n_m;
-                        M.flags = skip ? (1 | 16) : 1;
+                        M.flags = 1;
                         M.t.tau = hd.tau;
                         M.t.flA = hd.flA;
                         M.slab = slab;
@@ -779,7 +784,7 @@ __global__ void __launch_bounds__(kPairThreads, kPairCtas) pair_step_kernel(cons
         } else if (flags & 1) {                            // tile end: clamp (Q12), store, flag
             const int np = M.np, n_m = M.n_m;
             const int v = isB ? M.t.v0B + (r - kPairVB) : M.t.v0A + r;
-            const bool ok = !(flags & 16) && (!isB || M.hasB) && v >= 0 && v < M.n_v;   // 16: empty tile
+            const bool ok = (!isB || M.hasB) && v >= 0 && v < M.n_v;
             bool fin = false;
             if (ok) {
                 double *o = M.t.outA + (int64_t)(v - M.t.v0A) * M.rowlen + (isB ? M.slab : (int64_t)0);
