@@ -66,7 +66,8 @@ struct madpipe_ctx {
     // MADPIPE_AUX_GRID=t,f: persistent grids of t and f blocks per SM for the pair path's list
     // builder and fixup kernels (they run side by side on two streams; 0 = one block per item)
     int aux_grid_trans = 0, aux_grid_fix = 0;
-    int replay_pass = -1, replay_reps = 0, replay_diag = 0;   // MADPIPE_REPLAY=pass,reps,diag (diagnostic)
+    int replay_pass = -1, replay_reps = 0, replay_diag = 0;
+    int pass_timing = 0;      // MADPIPE_PASS_TIMING=1: per-pass step / fixup / list-builder / gap times to stderr   // MADPIPE_REPLAY=pass,reps,diag (diagnostic)
     int trans_overlap = 0;    // MADPIPE_TRANS_OVERLAP=1: pair path builds pass i+1's lists beside step(i) (measured
                               // slower at GPT: 909 vs 886 ms, 5% more entries kept unverified + contention)
     DevBuf profbuf;
@@ -279,7 +280,8 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, int32_t rank, i
     c->prof = pf && pf[0] == '1';
     if (const char *e = getenv("MADPIPE_NPROD")) c->n_prod = std::max(1, std::min(4, atoi(e)));
     if (const char *e = getenv("MADPIPE_TILE_BLOCK")) c->tile_block = std::max(1, atoi(e));
-    if (const char *e = getenv("MADPIPE_TRANS_OVERLAP")) c->trans_overlap = atoi(e) != 0;
+    if (const char *e = getenv("MADPIPE_TRANS_OVERLAP")) c->trans_overlap = std::max(0, std::min(2, atoi(e)));
+    if (const char *e = getenv("MADPIPE_PASS_TIMING")) c->pass_timing = atoi(e) != 0;
     if (const char *e = getenv("MADPIPE_REPLAY")) sscanf(e, "%d,%d,%d", &c->replay_pass, &c->replay_reps, &c->replay_diag);
     if (const char *e = getenv("MADPIPE_AUX_GRID")) {
         int t = 0, f = 0;
@@ -721,10 +723,18 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
             //   slabs <= l and, for slab l+1, a superset of what fixup(i) will flag (fix_slab).
             launch_pair_trans(djobs, nj, n_v_max, 1, nmp, 0, -1, INT_MAX, 0, ctx->stream);
             ctx->launches++;
+            // MADPIPE_PASS_TIMING (diagnostic): events before/after each step, after each fixup (main
+            // stream) and after each list build (aux stream)
+            std::vector<cudaEvent_t> pt;
+            const int n_pass = (maxL + 1) / 2;
+            if (ctx->pass_timing) {
+                pt.resize(4 * (size_t)n_pass);
+                for (auto &e : pt) cudaEventCreate(&e);
+            }
             for (int l = 1; l <= maxL; l += 2) {
                 const int i = l >> 1, b = i & 1;
-                if (i >= 1) CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->stream, ctx->ev_tr[b], 0));
-                if (ctx->trans_overlap && l + 2 <= maxL) {
+                if (i >= 1 && ctx->trans_overlap != 2) CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->stream, ctx->ev_tr[b], 0));
+                if (ctx->trans_overlap == 1 && l + 2 <= maxL) {
                     CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[b], ctx->stream));
                     CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_st[b], 0));
                     launch_pair_trans(djobs, nj, n_v_max, l + 2, nmp, (size_t)(b ^ 1) * list_buf_entries, -1, l,
@@ -754,27 +764,64 @@ int run_jobs(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vect
                     cudaEventDestroy(e1);
                 }
                 if (per_launch) cudaEventRecord(ctx->ev_pool[2 * n_rec], ctx->stream);
+                if (ctx->pass_timing) cudaEventRecord(pt[4 * i], ctx->stream);
                 launch_pair_step((const int2 *)ctx->tdesc.p, n_tiles, ctx->tlist.p, b * list_buf_entries, cap, nmp,
                                  p_np, nsg, persist_grid,
                                  (unsigned long long *)(ctx->prof ? ctx->profbuf.p : nullptr),
                                  ctx->stream);
                 if (per_launch) cudaEventRecord(ctx->ev_pool[2 * n_rec + 1], ctx->stream);
+                if (ctx->pass_timing) cudaEventRecord(pt[4 * i + 1], ctx->stream);
                 n_rec++;
                 ctx->launches++;
-                if (!ctx->trans_overlap && l + 2 <= maxL) {
+                if (ctx->trans_overlap == 0 && l + 2 <= maxL) {
                     CUDA_TRY(ctx, cudaEventRecord(ctx->ev_st[b], ctx->stream));
                     CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_st[b], 0));
                     launch_pair_trans(djobs, nj, n_v_max, l + 2, nmp, (size_t)(b ^ 1) * list_buf_entries, l + 1,
                                       INT_MAX, ctx->aux_grid_trans, ctx->aux);
                     CUDA_TRY(ctx, cudaEventRecord(ctx->ev_tr[b ^ 1], ctx->aux));
+                    if (ctx->pass_timing) cudaEventRecord(pt[4 * i + 3], ctx->aux);
                     ctx->launches++;
                 }
                 if (l + 1 <= maxL) {
                     launch_pair_fixup(djobs, nj, n_v_max, l + 1, nmp, ctx->aux_grid_fix, ctx->stream);
                     ctx->launches++;
                 }
+                if (ctx->pass_timing) cudaEventRecord(pt[4 * i + 2], ctx->stream);
+                if (ctx->trans_overlap == 2 && l + 2 <= maxL) {
+                    // serial: the lists of pass i+1 after fixup(i) on the same stream (every flag final)
+                    launch_pair_trans(djobs, nj, n_v_max, l + 2, nmp, (size_t)(b ^ 1) * list_buf_entries, -1, INT_MAX,
+                                      ctx->aux_grid_trans, ctx->stream);
+                    if (ctx->pass_timing) cudaEventRecord(pt[4 * i + 3], ctx->stream);
+                    ctx->launches++;
+                }
             }
             ctx->n_rec = n_rec;
+            if (ctx->pass_timing) {
+                cudaStreamSynchronize(ctx->stream);
+                cudaStreamSynchronize(ctx->aux);
+                double st = 0, fx = 0, tr = 0, gap = 0, crit = 0;
+                for (int q = 0; q < n_pass; q++) {
+                    float a = 0.f;
+                    cudaEventElapsedTime(&a, pt[4 * q], pt[4 * q + 1]);
+                    st += a;
+                    cudaEventElapsedTime(&a, pt[4 * q + 1], pt[4 * q + 2]);
+                    fx += a;
+                    if (2 * q + 3 <= maxL) {
+                        cudaEventElapsedTime(&a, pt[4 * q + 1], pt[4 * q + 3]);
+                        tr += a;
+                    }
+                    if (q + 1 < n_pass) {
+                        cudaEventElapsedTime(&a, pt[4 * q + 1], pt[4 * (q + 1)]);
+                        crit += a;
+                        cudaEventElapsedTime(&a, pt[4 * q + 2], pt[4 * (q + 1)]);
+                        gap += a;
+                    }
+                }
+                fprintf(stderr, "[madpipe pass timing] %d jobs, %d passes: step %.3f ms, step end -> fixup end %.3f ms, "
+                        "step end -> next lists built %.3f ms, step end -> next step start %.3f ms, fixup end -> next step "
+                        "start %.3f ms\n", nj, n_pass, st, fx, tr, crit, gap);
+                for (auto &e : pt) cudaEventDestroy(e);
+            }
         } else {
         if (kern == 2) {
             launch_window(djobs, nj, maxL, ctx->stream);
