@@ -302,6 +302,7 @@ __global__ void __launch_bounds__(64) trans_kernel(const Job *jobs, int l, int n
     unsigned live = 0, useful = 0;
     int n = 0;
     TransEntry *list = J.tlist + buf_off + (size_t)(row_ok ? v : 0) * J.code_cap;
+    const RowCtx rc = row_ctx(J, row_ok ? v : 0);
     for (int kb = kmin; kb <= l; kb += 16) {   // same trip count in both halves (same job, layer)
         const int k = kb + hl;
         int32_t tr = -1;
@@ -309,7 +310,7 @@ __global__ void __launch_bounds__(64) trans_kernel(const Job *jobs, int l, int n
         bool use = false;
         if (row_ok && k <= l) {
             Ukl = __dsub_rn(Ul, J.Up[k - 1]);
-            tr = transition(J, k, l, v, Ukl, nullptr);
+            tr = transition_rc(J, k, l, rc, Ukl, nullptr);
             if (tr >= 0) {
                 live++;
                 // a source row that is +inf everywhere can only contribute +inf (exact skip)

@@ -236,6 +236,7 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
     const int kA = J.kwin[l];                    // window starts max(kmin_tau, kmin_W)
     const int kw = isB ? (hasB ? J.kwin[l + 1] : l + 1) : kA;
     unsigned live = 0, useful = 0;
+    const RowCtx rc = row_ctx(J, row_ok ? v : 0);    // the row's k-invariant part of every transition
     // option k = l+1 of the layer-(l+1) rows, for pair_fixup_kernel: its transition
     // (or kSkip), one word per row, buffer (pass % 2) -- the fixup of this pass runs
     // while the next pass's lists are built
@@ -243,7 +244,7 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
         int32_t fx = kSkip;
         if (l + 1 >= kw) {
             int64_t d;
-            fx = transition(J, l + 1, l + 1, v, __dsub_rn(Ul1, Ul), &d);
+            fx = transition_rc(J, l + 1, l + 1, rc, __dsub_rn(Ul1, Ul), &d);
         }
         J.codes[(size_t)((l >> 1) & 1) * J.n_v + v] = fx;
     }
@@ -268,7 +269,7 @@ __device__ __forceinline__ void pair_trans_body(const Job &J, int vt, int lane, 
             code[u] = 0;
             if (row_ok && k <= l && k >= kw) {
                 int64_t d;
-                const int32_t tr = transition(J, k, lr, v, __dsub_rn(Ulr, J.Up[k - 1]), &d);
+                const int32_t tr = transition_rc(J, k, lr, rc, __dsub_rn(Ulr, J.Up[k - 1]), &d);
                 if (tr >= 0) {
                     live++;
                     key[u] = (k << 16) | (tr & 0xFFFF);

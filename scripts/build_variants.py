@@ -22,6 +22,8 @@ VARIANTS = {
     "l2pf6": "-DMP_PAIR_L2PF=6",                  # L2 prefetch 6 rounds ahead
     "l2pf2": "-DMP_PAIR_L2PF=2",
     "l2pf4": "-DMP_PAIR_L2PF=4",
+    "tminb6": "-DMP_TRANS_MINB=6",                # list builder compiled for 6 resident blocks per SM (80 registers)
+    "tminb4": "-DMP_TRANS_MINB=4",
     "ctas3": "-DMP_PAIR_CTAS=3",                  # 3 CTAs per SM (16-slot rings, <= 75 registers)
     # MADPIPE_REPLAY=pass,reps,diag honoured (diag 1: consumers skip the relaxation, 2: producer
     # skips the copies, 3: both) -- diagnostic replays only, never the solve itself
