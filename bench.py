@@ -426,8 +426,8 @@ def main():
     moved_rate = moved_step * K / (kern_ms / 1e3) / 1e9 if kern_ms > 0 and moved_step > 0 else None
     units = useful_step if useful_step > 0 else eff_step
     streaming = units / world * K * BYTES_PER_UPDATE / (kern_ms / 1e3) / 1e9 if kern_ms > 0 else None
-    traffic = _profile_json("r02_step_traffic.json") if args.config == "gpt" else None
-    pipes = _profile_json("r02_step_pipes.json") if args.config == "gpt" else None
+    traffic = _profile_json("r02b_step_traffic.json") if args.config == "gpt" else None
+    pipes = _profile_json("r02b_step_pipes.json") if args.config == "gpt" else None
     fp64 = _profile_json("r02_fp64_peak.json")
     n_launch = (cfg["L"] + 1) // 2 if not batch else None
     roof = {"bound": "hbm", "kernel": ctx.last_kernel(), "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",

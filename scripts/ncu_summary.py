@@ -2,7 +2,7 @@
 
     python scripts/ncu_summary.py launches <launches.csv> <out.md>
         per-kernel share of the device time from an `ncu --metrics gpu__time_duration.sum` launch list
-    python scripts/ncu_summary.py full <prof.ncu-rep> <out.md> [--pipes-json profiles/r02_step_pipes.json]
+    python scripts/ncu_summary.py full <prof.ncu-rep> <out.md> [--pipes-json profiles/r02b_step_pipes.json]
         key metrics + top stall reasons + hottest SASS lines of a `--set full` capture; the
         pipe utilisations of the (first) captured launch go to the JSON the bench reads
     python scripts/ncu_summary.py traffic <dram.csv> <one_solve.json> <out.json>

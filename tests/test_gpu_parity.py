@@ -425,3 +425,40 @@ def test_solve_dev_equals_solve_equals_oracle(ctx):
         d = {k: torch.from_numpy(np.ascontiguousarray(ch[k])).cuda() for k in ("uF", "uB", "W", "a")}
         ref = oracle.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
         _same_solution(ctx.solve_dev(d, P, M, beta, n_m, n_v, n_c, v_range=vr), ref)
+
+
+@pytest.mark.parametrize("env", [{"MADPIPE_TRANS_OVERLAP": "1"}, {"MADPIPE_TRANS_OVERLAP": "2"},
+                                 {"MADPIPE_AUX_GRID": "4,3"}])
+def test_pair_schedules(env):
+    """The two-layer path's alternative schedules of list building vs step and fixup
+    (lists of pass i+1 beside step(i) with unverified sources; after the fixup on one
+    stream; persistent list-builder / fixup grids) give the oracle's roots, tables and
+    solutions: the skip rules they use are supersets of the exact one."""
+    import os
+    old = {k: os.environ.get(k) for k in list(env) + ["MADPIPE_KERNEL"]}
+    os.environ.update(env)
+    os.environ["MADPIPE_KERNEL"] = "pair"
+    try:
+        c = mp.Context(0)
+    finally:
+        for k, v in old.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
+    try:
+        for ch, P, M, beta, n_m, n_v, n_c, vr in _comm_cases(6, 123):
+            ref = oracle.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr, n_threads=4)
+            tau, root = c.candidates(ch, P, M, beta, n_m, n_v, n_c, v_range=vr)
+            assert np.array_equal(root, ref["root"]), (P, n_m, n_v, vr)
+            _same_solution(c.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr), ref)
+            j = max(ref["cand_index"], 0)
+            A, _ = c.dp_table(ch, P, M, beta, n_m, n_v, n_c, j=j, v_range=vr)
+            A_ref, _, _ = oracle.table(ch, P, M, beta, n_m, n_v, vr, ref["tau"][j])
+            assert np.array_equal(A, A_ref)
+        cfg = configs.load("resnet50")
+        ch = chaingen.make(cfg["chain"])
+        got = c.solve(ch, *_args(cfg))
+        assert got["cand_index"] == cfg["oracle_cand_index"]
+    finally:
+        c.close()
