@@ -67,7 +67,8 @@ struct madpipe_ctx {
     // builder and fixup kernels (they run side by side on two streams; 0 = one block per item)
     int aux_grid_trans = 0, aux_grid_fix = 0;
     int replay_pass = -1, replay_reps = 0, replay_diag = 0;
-    int pass_timing = 0;      // MADPIPE_PASS_TIMING=1: per-pass step / fixup / list-builder / gap times to stderr   // MADPIPE_REPLAY=pass,reps,diag (diagnostic)
+    int pass_timing = 0;
+    int pair_min_p = 16;      // MADPIPE_PAIR_MIN_P: smallest P dispatched to the two-layer kernel      // MADPIPE_PASS_TIMING=1: per-pass step / fixup / list-builder / gap times to stderr   // MADPIPE_REPLAY=pass,reps,diag (diagnostic)
     int trans_overlap = 0;    // MADPIPE_TRANS_OVERLAP=1: pair path builds pass i+1's lists beside step(i) (measured
                               // slower at GPT: 909 vs 886 ms, 5% more entries kept unverified + contention)
     DevBuf profbuf;
@@ -282,6 +283,7 @@ extern "C" int madpipe_ctx_create(madpipe_ctx **out, int device, int32_t rank, i
     if (const char *e = getenv("MADPIPE_TILE_BLOCK")) c->tile_block = std::max(1, atoi(e));
     if (const char *e = getenv("MADPIPE_TRANS_OVERLAP")) c->trans_overlap = std::max(0, std::min(2, atoi(e)));
     if (const char *e = getenv("MADPIPE_PASS_TIMING")) c->pass_timing = atoi(e) != 0;
+    if (const char *e = getenv("MADPIPE_PAIR_MIN_P")) c->pair_min_p = std::max(2, atoi(e));
     if (const char *e = getenv("MADPIPE_REPLAY")) sscanf(e, "%d,%d,%d", &c->replay_pass, &c->replay_reps, &c->replay_diag);
     if (const char *e = getenv("MADPIPE_AUX_GRID")) {
         int t = 0, f = 0;
@@ -459,10 +461,11 @@ void tile_geom(int P, int n_v, int threads, int *vb, int *np, int *n_ptiles, int
 
 // Step kernel of a job (measured): the persistent TMA kernel moves one row
 // segment per stage, which pays off from ~1 KB segments; below, plain loads win; the
-// two-layer kernel where it measured faster: P > 33 at GPT shape (profiles/r01_pair_dispatch.md)
-// and, with its one-row-per-thread mode for tiles of <= 32 processors, from P = 17 on the
-// config-5 batch (profiles/r02_batch.md), n_mem <= 8.  MADPIPE_KERNEL forces one (falling
-// back where it does not apply).
+// two-layer kernel where it measured faster: P > 33 at GPT shape (profiles/r01_pair_dispatch.md),
+// with its one-row-per-thread mode for tiles of <= 32 processors from P = 17 on the config-5
+// batch (profiles/r02_batch.md), and from P = 16 in round 2b (Inception/VGG shapes 214 / 33 ms
+// vs 224 / 35 ms with the single-layer kernel, config 5 13.3 vs 13.7 s; MADPIPE_PAIR_MIN_P),
+// n_mem <= 8.  MADPIPE_KERNEL forces one (falling back where it does not apply).
 int step_kernel_for(const madpipe_ctx *ctx, int P, int nmp, int n_v, int all_maxL) {
     int k = ctx->kernel;
     if (k == 3 && !pair_supported(P, nmp, n_v, all_maxL)) k = -1;
@@ -470,7 +473,7 @@ int step_kernel_for(const madpipe_ctx *ctx, int P, int nmp, int n_v, int all_max
         int vb_, np_, npt_, nt_;
         persist_geom(P, n_v, nmp, &vb_, &np_, &npt_, &nt_);
         k = (np_ + 1) * nmp * 8 >= 1024 ? 2 : 0;
-        if (P > 16 && pair_supported(P, nmp, n_v, all_maxL)) k = 3;
+        if (P >= ctx->pair_min_p && pair_supported(P, nmp, n_v, all_maxL)) k = 3;
     }
     return k;
 }
