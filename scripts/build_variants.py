@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Build the compile-time A/B variants of libmadpipe as their own in-tree libraries
 (paper_conf_ipps_beaumontes22_b200/libmadpipe_<name>.so, flags stamped in <lib>.flags),
-for scripts/gpu_variants.sh.  Every variant must pass the pair-path parity tests before
+for scripts/gpu_ab.sh.  Every variant must pass the pair-path parity tests before
 it is timed; the defaults in the sources are the variants that won.
 
     python scripts/build_variants.py [name ...]      (default: all)
