@@ -428,24 +428,18 @@ def test_solve_dev_equals_solve_equals_oracle(ctx):
 
 
 @pytest.mark.parametrize("env", [{"MADPIPE_TRANS_OVERLAP": "1"}, {"MADPIPE_TRANS_OVERLAP": "2"},
-                                 {"MADPIPE_AUX_GRID": "4,3"}])
-def test_pair_schedules(env):
-    """The two-layer path's alternative schedules of list building vs step and fixup
-    (lists of pass i+1 beside step(i) with unverified sources; after the fixup on one
-    stream; persistent list-builder / fixup grids) give the oracle's roots, tables and
-    solutions: the skip rules they use are supersets of the exact one."""
-    import os
-    old = {k: os.environ.get(k) for k in list(env) + ["MADPIPE_KERNEL"]}
-    os.environ.update(env)
-    os.environ["MADPIPE_KERNEL"] = "pair"
-    try:
-        c = mp.Context(0)
-    finally:
-        for k, v in old.items():
-            if v is None:
-                os.environ.pop(k, None)
-            else:
-                os.environ[k] = v
+                                 {"MADPIPE_AUX_GRID": "4,3"}, {"MADPIPE_PAIR_ROUND": "1"},
+                                 {"MADPIPE_PAIR_ROUND": "16"}])
+def test_pair_schedules(env, monkeypatch):
+    """The two-layer path's alternative schedules -- list building vs step and fixup (lists
+    of pass i+1 beside step(i) with unverified sources; after the fixup on one stream;
+    persistent list-builder / fixup grids) and the producer's round size (one slot per
+    round: the queue protocol at its finest grain; 16 slots: most of the ring in flight) --
+    give the oracle's roots, tables and solutions."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)                 # read at context creation or at every launch
+    monkeypatch.setenv("MADPIPE_KERNEL", "pair")
+    c = mp.Context(0)
     try:
         for ch, P, M, beta, n_m, n_v, n_c, vr in _comm_cases(6, 123):
             ref = oracle.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr, n_threads=4)
