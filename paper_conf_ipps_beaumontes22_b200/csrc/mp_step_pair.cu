@@ -881,7 +881,7 @@ __device__ __forceinline__ void pair_fixup_body(const Job &J, int v, int lane, i
 }
 
 #ifndef MP_FIX_MINB
-#define MP_FIX_MINB 1
+#define MP_FIX_MINB 8
 #endif
 __global__ void __launch_bounds__(128, MP_FIX_MINB) pair_fixup_kernel(const Job *jobs, int l1, int nmp, int xb,
                                                                        int n_items) {
