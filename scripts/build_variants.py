@@ -24,9 +24,7 @@ VARIANTS = {
     "l2pf4": "-DMP_PAIR_L2PF=4",
     "tminb6": "-DMP_TRANS_MINB=6",                # list builder compiled for 6 resident blocks per SM (80 registers)
     "tminb4": "-DMP_TRANS_MINB=4",
-    "fixminb8": "-DMP_FIX_MINB=8",                # fixup compiled for 8 resident blocks per SM (64 registers)
-    "fixminb8fb8": "-DMP_FIX_MINB=8 -DMP_FIX_FB=8",
-    "fixminb6": "-DMP_FIX_MINB=6",
+    "fixminb1": "-DMP_FIX_MINB=1",                # fixup without a residency target (72 registers, 7 blocks per SM)
     "ctas3": "-DMP_PAIR_CTAS=3",                  # 3 CTAs per SM (16-slot rings, <= 75 registers)
     # MADPIPE_REPLAY=pass,reps,diag honoured (diag 1: consumers skip the relaxation, 2: producer
     # skips the copies, 3: both) -- diagnostic replays only, never the solve itself
