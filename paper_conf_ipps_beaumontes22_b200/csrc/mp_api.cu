@@ -973,6 +973,59 @@ struct TraceHook : BatchHook {
     }
 };
 
+// madpipe_alloc of candidate j from its traceback (period = tau_j, Q16)
+void fill_from_trace(madpipe_alloc *o, int32_t j, double tau, const TraceOut &t, const int32_t *st, int stride) {
+    o->period = tau;
+    o->load_period = t.load_period;
+    o->special_load = t.special_load;
+    o->cand_index = j;
+    o->n_stages = t.n_stages;
+    for (int s = 0; s < t.n_stages; s++) {
+        if (o->stage_first) o->stage_first[s] = st[s];
+        if (o->stage_last) o->stage_last[s] = st[stride + s];
+        if (o->stage_proc) o->stage_proc[s] = st[2 * stride + s];
+    }
+}
+
+// One-rank sweeps (a8 without the re-solve): after each batch, the smallest feasible
+// candidate found so far is traced back straight from the batch's tables, before they are
+// reused.  Candidates run in ascending order, so the batch holding the final winner traces
+// it.  jl_dev is the sweep's device int32 (one chain).
+struct SweepTraceHook : BatchHook {
+    int nmp = 0, stride = 1;
+    const std::vector<JobSpec> *js = nullptr;   // the job list of the current run_jobs call
+    const int32_t *jl_dev = nullptr;
+    int32_t best = INT32_MAX;                   // the candidate traced so far
+    TraceOut out{};
+    std::vector<int32_t> stages;
+    double tau = 0.0;
+    int after_batch(madpipe_ctx *ctx, const std::vector<int> &ids, Job *jobs_dev) override {
+        int32_t jl = INT32_MAX;
+        CUDA_TRY(ctx, d2h(ctx, &jl, jl_dev, sizeof(int32_t)));
+        CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+        if (jl >= best) return MADPIPE_OK;
+        for (size_t i = 0; i < ids.size(); i++) {
+            if ((*js)[ids[i]].j != jl) continue;
+            CUDA_TRY(ctx, ctx->trace.ensure(sizeof(TraceOut)));
+            CUDA_TRY(ctx, ctx->stages.ensure(sizeof(int32_t) * 3 * (size_t)stride));
+            launch_traceback(jobs_dev + i, 1, nmp, (TraceOut *)ctx->trace.p, (int32_t *)ctx->stages.p, stride,
+                             ctx->stream);
+            ctx->launches++;
+            CUDA_TRY(ctx, cudaGetLastError());
+            Job jb;
+            stages.resize(3 * (size_t)stride);
+            CUDA_TRY(ctx, d2h(ctx, &out, ctx->trace.p, sizeof(TraceOut)));
+            CUDA_TRY(ctx, d2h(ctx, stages.data(), ctx->stages.p, sizeof(int32_t) * stages.size()));
+            CUDA_TRY(ctx, d2h(ctx, &jb, jobs_dev + i, sizeof(Job)));
+            CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+            tau = jb.tau;
+            best = jl;
+            break;
+        }
+        return MADPIPE_OK;
+    }
+};
+
 void fill_infeasible(madpipe_alloc *out, int64_t cu) {
     out->period = INFINITY;
     out->load_period = INFINITY;
@@ -1022,17 +1075,7 @@ int resolve_impl(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::
         if (t.status != 0)
             return fail(ctx, MADPIPE_ESTATE, "resolve of candidate %d: %s", js[i].j,
                         t.status == 1 ? "root is infeasible" : "traceback found no decision");
-        o->period = hook.taus[i];
-        o->load_period = t.load_period;
-        o->special_load = t.special_load;
-        o->cand_index = js[i].j;
-        o->n_stages = t.n_stages;
-        const int32_t *st = hook.stages.data() + i * 3 * (size_t)maxL;
-        for (int s = 0; s < t.n_stages; s++) {
-            if (o->stage_first) o->stage_first[s] = st[s];
-            if (o->stage_last) o->stage_last[s] = st[maxL + s];
-            if (o->stage_proc) o->stage_proc[s] = st[2 * maxL + s];
-        }
+        fill_from_trace(o, js[i].j, hook.taus[i], t, hook.stages.data() + i * 3 * (size_t)maxL, maxL);
     }
     return MADPIPE_OK;
 }
@@ -1098,6 +1141,11 @@ int solve_common(madpipe_ctx *ctx, const madpipe_chain *chain, bool on_device, i
     int64_t cu = 0;
     int32_t jstar = INT32_MAX;
     const int R = ctx->rank, W = ctx->world;
+    // one rank: the winner is traced back from its sweep batch (no re-solve)
+    SweepTraceHook th;
+    th.nmp = nmp_of(disc->n_mem);
+    th.stride = std::max(1, (int)chain->L);
+    th.jl_dev = (const int32_t *)ctx->jl.p;
     // One round: this rank evaluates its share of `js` (ascending; with `early`, it stops
     // at its first feasible candidate -- exact, a smaller feasible index always wins),
     // then the ranks min-reduce their smallest feasible index (a7, one all-reduce).
@@ -1109,8 +1157,9 @@ int solve_common(madpipe_ctx *ctx, const madpipe_chain *chain, bool on_device, i
         for (size_t i = (size_t)R; i < js.size(); i += (size_t)W) mine.push_back(js[i]);
         std::vector<uint64_t> counts;
         if (!mine.empty()) {
-            r = run_jobs(ctx, cs, cd, disc, mine, (int32_t *)ctx->jl.p, nullptr, nullptr, &counts, early, nullptr,
-                         true);
+            th.js = &mine;
+            r = run_jobs(ctx, cs, cd, disc, mine, (int32_t *)ctx->jl.p, nullptr, nullptr, &counts, early,
+                         W == 1 ? &th : nullptr, true);
             if (r) return r;
             for (auto x : counts) cu += (int64_t)x;
             *ms_acc += ctx->sweep_ms; *kern_acc += ctx->step_ms;
@@ -1158,7 +1207,16 @@ int solve_common(madpipe_ctx *ctx, const madpipe_chain *chain, bool on_device, i
         fill_infeasible(out, cu);
         return MADPIPE_INFEASIBLE;
     }
-    // a8: every rank re-solves the winner and traces it back (deterministic: no broadcast)
+    // a8: one rank traced the winner in its sweep batch; at N ranks every rank re-solves the
+    // winner and traces it back (deterministic: no broadcast)
+    if (W == 1 && th.best == jstar) {
+        if (th.out.status != 0)
+            return fail(ctx, MADPIPE_ESTATE, "traceback of candidate %d: %s", jstar,
+                        th.out.status == 1 ? "root is infeasible" : "traceback found no decision");
+        fill_from_trace(out, jstar, th.tau, th.out, th.stages.data(), th.stride);
+        out->cell_updates = cu;
+        return MADPIPE_OK;
+    }
     std::vector<int32_t> js{jstar};
     rc = resolve_impl(ctx, cs, cd, disc, js, out);
     out->cell_updates = cu;
