@@ -987,40 +987,59 @@ void fill_from_trace(madpipe_alloc *o, int32_t j, double tau, const TraceOut &t,
     }
 }
 
-// One-rank sweeps (a8 without the re-solve): after each batch, the smallest feasible
-// candidate found so far is traced back straight from the batch's tables, before they are
-// reused.  Candidates run in ascending order, so the batch holding the final winner traces
-// it.  jl_dev is the sweep's device int32 (one chain).
+// One-rank sweeps (a8 without the re-solve): after each batch, every chain's smallest
+// feasible candidate found so far is traced back straight from the batch's tables, before
+// they are reused.  A chain's candidates run in ascending order (batch_sweep keeps them
+// candidate-major), so the batch holding its final winner traces it.  jl_dev: the sweep's
+// device int32[n_chains].
 struct SweepTraceHook : BatchHook {
-    int nmp = 0, stride = 1;
+    int nmp = 0, stride = 1, n_chains = 0;
     const std::vector<JobSpec> *js = nullptr;   // the job list of the current run_jobs call
     const int32_t *jl_dev = nullptr;
-    int32_t best = INT32_MAX;                   // the candidate traced so far
-    TraceOut out{};
-    std::vector<int32_t> stages;
-    double tau = 0.0;
+    std::vector<int32_t> best;                  // per chain: the candidate traced so far
+    std::vector<TraceOut> outs;
+    std::vector<int32_t> stages;                // [chain][3][stride]
+    std::vector<double> taus;
+    void init(int n, int nmp_, int stride_, const int32_t *jl) {
+        n_chains = n; nmp = nmp_; stride = std::max(1, stride_); jl_dev = jl;
+        best.assign(n, INT32_MAX);
+        outs.assign(n, TraceOut{});
+        stages.assign(3 * (size_t)stride * n, 0);
+        taus.assign(n, 0.0);
+    }
     int after_batch(madpipe_ctx *ctx, const std::vector<int> &ids, Job *jobs_dev) override {
-        int32_t jl = INT32_MAX;
-        CUDA_TRY(ctx, d2h(ctx, &jl, jl_dev, sizeof(int32_t)));
+        std::vector<int32_t> jl(n_chains);
+        CUDA_TRY(ctx, d2h(ctx, jl.data(), jl_dev, sizeof(int32_t) * n_chains));
         CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
-        if (jl >= best) return MADPIPE_OK;
+        std::vector<int> sel;                   // batch positions of newly found winners
         for (size_t i = 0; i < ids.size(); i++) {
-            if ((*js)[ids[i]].j != jl) continue;
-            CUDA_TRY(ctx, ctx->trace.ensure(sizeof(TraceOut)));
-            CUDA_TRY(ctx, ctx->stages.ensure(sizeof(int32_t) * 3 * (size_t)stride));
-            launch_traceback(jobs_dev + i, 1, nmp, (TraceOut *)ctx->trace.p, (int32_t *)ctx->stages.p, stride,
-                             ctx->stream);
+            const JobSpec &s = (*js)[ids[i]];
+            if (s.j == jl[s.chain] && jl[s.chain] < best[s.chain]) sel.push_back((int)i);
+        }
+        if (sel.empty()) return MADPIPE_OK;
+        const int K = (int)sel.size(), nj = (int)ids.size();
+        CUDA_TRY(ctx, ctx->trace.ensure(sizeof(TraceOut) * K));
+        CUDA_TRY(ctx, ctx->stages.ensure(sizeof(int32_t) * 3 * (size_t)stride * K));
+        for (int k = 0; k < K; k++) {
+            launch_traceback(jobs_dev + sel[k], 1, nmp, (TraceOut *)ctx->trace.p + k,
+                             (int32_t *)ctx->stages.p + 3 * (size_t)stride * k, stride, ctx->stream);
             ctx->launches++;
-            CUDA_TRY(ctx, cudaGetLastError());
-            Job jb;
-            stages.resize(3 * (size_t)stride);
-            CUDA_TRY(ctx, d2h(ctx, &out, ctx->trace.p, sizeof(TraceOut)));
-            CUDA_TRY(ctx, d2h(ctx, stages.data(), ctx->stages.p, sizeof(int32_t) * stages.size()));
-            CUDA_TRY(ctx, d2h(ctx, &jb, jobs_dev + i, sizeof(Job)));
-            CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
-            tau = jb.tau;
-            best = jl;
-            break;
+        }
+        CUDA_TRY(ctx, cudaGetLastError());
+        std::vector<TraceOut> o(K);
+        std::vector<int32_t> st(3 * (size_t)stride * K);
+        std::vector<Job> jb(nj);
+        CUDA_TRY(ctx, d2h(ctx, o.data(), ctx->trace.p, sizeof(TraceOut) * K));
+        CUDA_TRY(ctx, d2h(ctx, st.data(), ctx->stages.p, sizeof(int32_t) * st.size()));
+        CUDA_TRY(ctx, d2h(ctx, jb.data(), jobs_dev, sizeof(Job) * nj));
+        CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+        for (int k = 0; k < K; k++) {
+            const int c = (*js)[ids[sel[k]]].chain;
+            outs[c] = o[k];
+            taus[c] = jb[sel[k]].tau;
+            best[c] = jl[c];
+            std::copy(st.begin() + 3 * (size_t)stride * k, st.begin() + 3 * (size_t)stride * (k + 1),
+                      stages.begin() + 3 * (size_t)stride * c);
         }
         return MADPIPE_OK;
     }
@@ -1143,9 +1162,7 @@ int solve_common(madpipe_ctx *ctx, const madpipe_chain *chain, bool on_device, i
     const int R = ctx->rank, W = ctx->world;
     // one rank: the winner is traced back from its sweep batch (no re-solve)
     SweepTraceHook th;
-    th.nmp = nmp_of(disc->n_mem);
-    th.stride = std::max(1, (int)chain->L);
-    th.jl_dev = (const int32_t *)ctx->jl.p;
+    th.init(1, nmp_of(disc->n_mem), (int)chain->L, (const int32_t *)ctx->jl.p);
     // One round: this rank evaluates its share of `js` (ascending; with `early`, it stops
     // at its first feasible candidate -- exact, a smaller feasible index always wins),
     // then the ranks min-reduce their smallest feasible index (a7, one all-reduce).
@@ -1209,11 +1226,11 @@ int solve_common(madpipe_ctx *ctx, const madpipe_chain *chain, bool on_device, i
     }
     // a8: one rank traced the winner in its sweep batch; at N ranks every rank re-solves the
     // winner and traces it back (deterministic: no broadcast)
-    if (W == 1 && th.best == jstar) {
-        if (th.out.status != 0)
+    if (W == 1 && th.best[0] == jstar) {
+        if (th.outs[0].status != 0)
             return fail(ctx, MADPIPE_ESTATE, "traceback of candidate %d: %s", jstar,
-                        th.out.status == 1 ? "root is infeasible" : "traceback found no decision");
-        fill_from_trace(out, jstar, th.tau, th.out, th.stages.data(), th.stride);
+                        th.outs[0].status == 1 ? "root is infeasible" : "traceback found no decision");
+        fill_from_trace(out, jstar, th.taus[0], th.outs[0], th.stages.data(), th.stride);
         out->cell_updates = cu;
         return MADPIPE_OK;
     }
@@ -1317,7 +1334,7 @@ int prepare_batch(madpipe_ctx *ctx, int32_t n, const madpipe_chain *chains, cons
 // c among the jobs this rank owns (INT32_MAX if none); cu[c] <- this rank's cell-updates.
 int batch_sweep(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::vector<ChainDev> &cd,
                 const madpipe_disc *disc, int rank, int world, const std::vector<int32_t> &owner,
-                std::vector<int64_t> &cu) {
+                std::vector<int64_t> &cu, SweepTraceHook *th = nullptr) {
     const int n = (int)cs.size(), n_c = disc->n_periods;
     CUDA_TRY(ctx, ctx->jl.ensure(sizeof(int32_t) * n));
     { int _r = fill_int_max(ctx, (int32_t *)ctx->jl.p, n); if (_r) return _r; }
@@ -1342,8 +1359,14 @@ int batch_sweep(madpipe_ctx *ctx, const std::vector<ChainSpec> &cs, const std::v
     cu.assign(n, 0);
     if (js.empty()) return MADPIPE_OK;
     std::vector<uint64_t> counts;
+    if (th) {
+        int maxL = 1;
+        for (const auto &c : cs) maxL = std::max(maxL, (int)c.c.L);
+        th->init(n, nmp, maxL, (const int32_t *)ctx->jl.p);
+        th->js = &js;
+    }
     int rc = run_jobs(ctx, cs, cd, disc, js, (int32_t *)ctx->jl.p, nullptr, nullptr, &counts,
-                      disc->early_exit != 0, nullptr, true);
+                      disc->early_exit != 0, th, true);
     if (rc) return rc;
     for (size_t i = 0; i < js.size(); i++) cu[js[i].chain] += (int64_t)counts[i];
     return MADPIPE_OK;
@@ -1477,7 +1500,9 @@ extern "C" int madpipe_solve_batch(madpipe_ctx *ctx, int32_t n, const madpipe_ch
     rc = upload_chains(ctx, cs, cd);
     if (rc) return rc;
     std::vector<int64_t> cu;
-    rc = batch_sweep(ctx, cs, cd, disc, R, W, owner, cu);
+    SweepTraceHook th;                            // one rank: winners traced in their sweep batches
+    const bool one = W == 1 && !ctx->comm;
+    rc = batch_sweep(ctx, cs, cd, disc, R, W, owner, cu, one ? &th : nullptr);
     if (rc) return rc;
     rc = allreduce_min(ctx, (int32_t *)ctx->jl.p, (size_t)n);     // a7 over int32[n]
     if (rc) return rc;
@@ -1485,11 +1510,30 @@ extern "C" int madpipe_solve_batch(madpipe_ctx *ctx, int32_t n, const madpipe_ch
     CUDA_TRY(ctx, d2h(ctx, jstar.data(), ctx->jl.p, sizeof(int32_t) * n));
     CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
     for (int i = 0; i < n; i++) fill_infeasible(&out[i], cu[i]);
-    if (W == 1 && !ctx->comm) {
-        std::vector<int32_t> all(n, 0);
-        rc = batch_resolve(ctx, cs, cd, disc, jstar, all, 0, out);
+    if (one) {
+        // winners traced during the sweep; anything else (none expected) is re-solved
+        std::vector<int32_t> rest(n, INT32_MAX);
+        bool any = false;
+        for (int c = 0; c < n; c++) {
+            if (jstar[c] == INT32_MAX) continue;
+            if (th.best.size() == (size_t)n && th.best[c] == jstar[c]) {
+                if (th.outs[c].status != 0)
+                    return fail(ctx, MADPIPE_ESTATE, "traceback of chain %d candidate %d: %s", c, jstar[c],
+                                th.outs[c].status == 1 ? "root is infeasible" : "traceback found no decision");
+                fill_from_trace(&out[c], jstar[c], th.taus[c], th.outs[c],
+                                th.stages.data() + 3 * (size_t)th.stride * c, th.stride);
+            } else {
+                rest[c] = jstar[c];
+                any = true;
+            }
+        }
+        if (any) {
+            std::vector<int32_t> all(n, 0);
+            rc = batch_resolve(ctx, cs, cd, disc, rest, all, 0, out);
+            if (rc) return rc;
+        }
         for (int i = 0; i < n; i++) out[i].cell_updates = cu[i];
-        return rc;
+        return MADPIPE_OK;
     }
     // each winner is re-solved by its owner, then one all-gather of fixed-size records
     std::vector<int32_t> rowner;
