@@ -456,3 +456,30 @@ def test_pair_schedules(env, monkeypatch):
         assert got["cand_index"] == cfg["oracle_cand_index"]
     finally:
         c.close()
+
+
+@pytest.mark.parametrize("kernel", ["pair", "persist", "v1"])
+def test_winner_traced_in_a_later_batch(kernel, monkeypatch):
+    """One-rank solves trace the winner straight from the sweep batch that found it (no
+    re-solve).  A table budget of one job per batch puts the winner in a later batch than the
+    first, for the full sweep and for early exit; allocations equal the oracle's and pass
+    the simulator, and the single-batch context agrees."""
+    monkeypatch.setenv("MADPIPE_KERNEL", kernel)
+    tiny = mp.Context(0, mem_budget=1)            # every batch: a single job
+    big = mp.Context(0)
+    try:
+        n_checked = 0
+        for ch, P, M, beta, n_m, n_v, n_c, vr in _comm_cases(12, 321):
+            ref = oracle.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr, n_threads=4)
+            if ref["rc"] != 0 or ref["cand_index"] < 1:
+                continue
+            for early in (False, True):
+                got = tiny.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr, early_exit=early)
+                _same_solution(got, ref)
+                _verify(ch, P, M, beta, got)
+                _same_solution(big.solve(ch, P, M, beta, n_m, n_v, n_c, v_range=vr, early_exit=early), ref)
+            n_checked += 1
+        assert n_checked >= 3, n_checked
+    finally:
+        tiny.close()
+        big.close()
