@@ -1,4 +1,4 @@
-# Round-2 GPU evidence (run through gpurun from the repo root).  STAGES selects parts:
+# GPU evidence (run through gpurun from the repo root; profiles/r02b_* came from STAGES="test bench prof").  STAGES selects parts:
 #   test   : build, smoke(), pytest -m gpu
 #   bench  : bench.py gpt (N=1), gpt through the N-GPU code path (torchrun world 1, ctx-owned
 #            NCCL communicator), batch config, CNN configs
